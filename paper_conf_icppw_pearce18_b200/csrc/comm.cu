@@ -1,0 +1,202 @@
+// comm.cu -- see comm.h.  NCCL transport for ranks > 1.
+#include <nccl.h>
+
+#include <cstring>
+
+#include "comm.h"
+
+namespace hydro {
+
+namespace {
+
+struct SlabDesc {   // one remote slab: which local domain, which global boxes, buffer offset
+  int32_t slot;     // local domain slot (source when packing, destination when unpacking)
+  int32_t peer;     // remote rank
+  int64_t nlo[3], nhi[3], zlo[3], zhi[3];
+  int64_t offset;   // in doubles, into the send or receive buffer
+  int64_t count;    // doubles: 6 * nodes + zones
+};
+
+__global__ void k_pack(const DomView *views, const SlabDesc *descs, double *buf, int unpack) {
+  const SlabDesc p = descs[blockIdx.y];
+  const DomView &D = views[p.slot];
+  double *b = buf + p.offset;
+  const int64_t nx = p.nhi[0] - p.nlo[0], ny = p.nhi[1] - p.nlo[1], nz = p.nhi[2] - p.nlo[2];
+  const int64_t nn = nx * ny * nz;
+  double *arr[6] = {D.xn, D.yn, D.zn, D.un, D.vn, D.wn};
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nn;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = t % nx, bb = (t / nx) % ny, c = t / (nx * ny);
+    const int64_t id = D.nid((int)(p.nlo[0] + a - D.lo[0]), (int)(p.nlo[1] + bb - D.lo[1]),
+                             (int)(p.nlo[2] + c - D.lo[2]));
+#pragma unroll
+    for (int f = 0; f < 6; ++f) {
+      if (unpack) arr[f][id] = b[f * nn + t];
+      else b[f * nn + t] = arr[f][id];
+    }
+  }
+  const int64_t zx = p.zhi[0] - p.zlo[0], zy = p.zhi[1] - p.zlo[1], zz = p.zhi[2] - p.zlo[2];
+  const int64_t nzn = zx * zy * zz;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nzn;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = t % zx, bb = (t / zx) % zy, c = t / (zx * zy);
+    const int64_t id = D.zid((int)(p.zlo[0] + a - D.lo[0]), (int)(p.zlo[1] + bb - D.lo[1]),
+                             (int)(p.zlo[2] + c - D.lo[2]));
+    if (unpack) D.en[id] = b[6 * nn + t];
+    else b[6 * nn + t] = D.en[id];
+  }
+}
+
+}  // namespace
+
+struct Comm {
+  ncclComm_t nccl = nullptr;
+  int rank = 0, nranks = 1;
+  std::vector<SlabDesc> sends, recvs;  // in global pair order
+  SlabDesc *sends_dev = nullptr, *recvs_dev = nullptr;
+  double *sendbuf = nullptr, *recvbuf = nullptr;
+  int64_t send_total = 0, recv_total = 0;
+  DomView *views_dev[2] = {nullptr, nullptr};
+  int *status_dev = nullptr;
+};
+
+int comm_unique_id(void *out128) {
+  static_assert(sizeof(ncclUniqueId) == 128, "NCCL unique id size");
+  ncclUniqueId id;
+  if (ncclGetUniqueId(&id) != ncclSuccess) return HYDRO_ENCCL;
+  std::memcpy(out128, &id, sizeof(id));
+  return HYDRO_OK;
+}
+
+int comm_create(Comm **out, const hydro_config *cfg, const Layout &L,
+                const std::vector<HaloPair> &remote, const std::vector<int32_t> &slot_of_dom,
+                void *, cudaStream_t s, std::string *err) {
+  if (!cfg->comm_id) {
+    *err = "nranks > 1 needs comm_id";
+    return HYDRO_EINVAL;
+  }
+  Comm *c = new Comm();
+  *out = c;
+  c->rank = cfg->rank;
+  c->nranks = cfg->nranks;
+  ncclUniqueId id;
+  std::memcpy(&id, cfg->comm_id, sizeof(id));
+  if (ncclCommInitRank(&c->nccl, cfg->nranks, id, cfg->rank) != ncclSuccess) {
+    *err = "ncclCommInitRank failed";
+    return HYDRO_ENCCL;
+  }
+  for (const HaloPair &P : remote) {
+    SlabDesc d;
+    for (int a = 0; a < 3; ++a) {
+      d.nlo[a] = P.nlo[a]; d.nhi[a] = P.nhi[a]; d.zlo[a] = P.zlo[a]; d.zhi[a] = P.zhi[a];
+    }
+    int64_t nn = 1, nz = 1;
+    for (int a = 0; a < 3; ++a) {
+      nn *= P.nhi[a] - P.nlo[a];
+      nz *= P.zhi[a] - P.zlo[a];
+    }
+    d.count = 6 * nn + nz;
+    if (slot_of_dom[P.src] >= 0) {  // we own the source: send
+      d.slot = slot_of_dom[P.src];
+      d.peer = L.dom[P.dst].rank;
+      d.offset = c->send_total;
+      c->send_total += d.count;
+      c->sends.push_back(d);
+    } else {  // we own the destination: receive
+      d.slot = slot_of_dom[P.dst];
+      d.peer = L.dom[P.src].rank;
+      d.offset = c->recv_total;
+      c->recv_total += d.count;
+      c->recvs.push_back(d);
+    }
+  }
+  auto ck = [&](cudaError_t e) {
+    if (e != cudaSuccess) *err = cudaGetErrorString(e);
+    return e == cudaSuccess;
+  };
+  if (!ck(cudaMalloc(&c->status_dev, sizeof(int)))) return HYDRO_ECUDA;
+  if (c->send_total) {
+    if (!ck(cudaMalloc(&c->sendbuf, c->send_total * sizeof(double)))) return HYDRO_ENOMEM;
+    if (!ck(cudaMalloc(&c->sends_dev, c->sends.size() * sizeof(SlabDesc)))) return HYDRO_ENOMEM;
+    if (!ck(cudaMemcpyAsync(c->sends_dev, c->sends.data(), c->sends.size() * sizeof(SlabDesc),
+                            cudaMemcpyHostToDevice, s)))
+      return HYDRO_ECUDA;
+  }
+  if (c->recv_total) {
+    if (!ck(cudaMalloc(&c->recvbuf, c->recv_total * sizeof(double)))) return HYDRO_ENOMEM;
+    if (!ck(cudaMalloc(&c->recvs_dev, c->recvs.size() * sizeof(SlabDesc)))) return HYDRO_ENOMEM;
+    if (!ck(cudaMemcpyAsync(c->recvs_dev, c->recvs.data(), c->recvs.size() * sizeof(SlabDesc),
+                            cudaMemcpyHostToDevice, s)))
+      return HYDRO_ECUDA;
+  }
+  return HYDRO_OK;
+}
+
+int comm_bind_views(Comm *c, const DomView *const *v0, const DomView *const *v1, int n,
+                    std::string *err) {
+  for (int p = 0; p < 2; ++p) {
+    std::vector<DomView> vv;
+    for (int i = 0; i < n; ++i) vv.push_back(*(p ? v1[i] : v0[i]));
+    if (cudaMalloc(&c->views_dev[p], sizeof(DomView) * (n ? n : 1)) != cudaSuccess) {
+      *err = "cudaMalloc views";
+      return HYDRO_ENOMEM;
+    }
+    if (n && cudaMemcpy(c->views_dev[p], vv.data(), sizeof(DomView) * n,
+                        cudaMemcpyHostToDevice) != cudaSuccess) {
+      *err = "cudaMemcpy views";
+      return HYDRO_ECUDA;
+    }
+  }
+  return HYDRO_OK;
+}
+
+int comm_dt_min(Comm *c, unsigned long long *dev_bits, cudaStream_t s) {
+  if (ncclAllReduce(dev_bits, dev_bits, 1, ncclUint64, ncclMin, c->nccl, s) != ncclSuccess)
+    return HYDRO_ENCCL;
+  return HYDRO_OK;
+}
+
+int comm_halo(Comm *c, int par, cudaStream_t s) {
+  if (!c->sends.empty())
+    k_pack<<<dim3(8, (unsigned)c->sends.size()), 256, 0, s>>>(c->views_dev[par], c->sends_dev,
+                                                              c->sendbuf, 0);
+  if (ncclGroupStart() != ncclSuccess) return HYDRO_ENCCL;
+  // Every rank walks the global pair list in the same order, so sends and receives between a
+  // pair of ranks match one to one.
+  for (const SlabDesc &d : c->sends)
+    if (ncclSend(c->sendbuf + d.offset, d.count, ncclFloat64, d.peer, c->nccl, s) != ncclSuccess)
+      return HYDRO_ENCCL;
+  for (const SlabDesc &d : c->recvs)
+    if (ncclRecv(c->recvbuf + d.offset, d.count, ncclFloat64, d.peer, c->nccl, s) != ncclSuccess)
+      return HYDRO_ENCCL;
+  if (ncclGroupEnd() != ncclSuccess) return HYDRO_ENCCL;
+  if (!c->recvs.empty())
+    k_pack<<<dim3(8, (unsigned)c->recvs.size()), 256, 0, s>>>(c->views_dev[par], c->recvs_dev,
+                                                              c->recvbuf, 1);
+  return cudaGetLastError() == cudaSuccess ? HYDRO_OK : HYDRO_ECUDA;
+}
+
+int comm_status_agree(Comm *c, int status) {
+  int v = status;
+  cudaMemcpy(c->status_dev, &v, sizeof(int), cudaMemcpyHostToDevice);
+  if (ncclAllReduce(c->status_dev, c->status_dev, 1, ncclInt32, ncclMin, c->nccl, 0) !=
+      ncclSuccess)
+    return HYDRO_ENCCL;
+  cudaMemcpy(&v, c->status_dev, sizeof(int), cudaMemcpyDeviceToHost);
+  return v;
+}
+
+void comm_destroy(Comm *c) {
+  if (!c) return;
+  if (c->nccl) ncclCommDestroy(c->nccl);
+  cudaFree(c->sendbuf);
+  cudaFree(c->recvbuf);
+  cudaFree(c->sends_dev);
+  cudaFree(c->recvs_dev);
+  cudaFree(c->views_dev[0]);
+  cudaFree(c->views_dev[1]);
+  cudaFree(c->status_dev);
+  delete c;
+}
+
+}  // namespace hydro

@@ -1,0 +1,36 @@
+// comm.h -- inter-rank communication of the cycle (one process per GPU): the ghost-layer halo
+// exchange with neighbouring domains on other ranks ("halo exchange" between
+// neighbouring domains; L513-520: the paper routed it through the host, GPU-direct was future
+// work) and the global dt min-reduction (S9).  Transport: NCCL 2.28 over NVLink/NVSwitch,
+// grouped ncclSend/ncclRecv for the halo, ncclAllReduce(min, uint64) on the bit pattern of the
+// non-negative dt (bit order == numeric order for non-negative doubles).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <string>
+#include <vector>
+
+#include "device.cuh"
+#include "layout.h"
+
+namespace hydro {
+
+struct Comm;
+
+int comm_unique_id(void *out128);
+// remote: halo pairs with exactly one local end (dst or src on this rank).
+int comm_create(Comm **out, const hydro_config *cfg, const Layout &L,
+                const std::vector<HaloPair> &remote, const std::vector<int32_t> &slot_of_dom,
+                void *unused, cudaStream_t s, std::string *err);
+// views_p[slot] = &DomView of parity p for every local domain slot (kept by pointer).
+int comm_bind_views(Comm *c, const DomView *const *views0, const DomView *const *views1, int n,
+                    std::string *err);
+// In-place global min of a device uint64 (dt bits).
+int comm_dt_min(Comm *c, unsigned long long *dev_bits, cudaStream_t s);
+// Exchange the next-parity ghost slabs of parity-`par` views with remote neighbours.
+int comm_halo(Comm *c, int par, cudaStream_t s);
+// Agree on a status code across ranks (the most negative wins).
+int comm_status_agree(Comm *c, int status);
+void comm_destroy(Comm *c);
+
+}  // namespace hydro

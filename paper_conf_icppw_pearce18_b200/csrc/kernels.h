@@ -1,0 +1,44 @@
+// kernels.h -- host-side launchers for the CUDA kernels (all enqueue on `s`, never synchronise).
+#pragma once
+#include <cuda_runtime.h>
+
+#include "device.cuh"
+
+namespace hydro {
+
+struct HaloCopy {  // one intra-GPU ghost slab copy (global boxes, half-open)
+  int32_t dst, src;  // local domain slots
+  int64_t nlo[3], nhi[3], zlo[3], zhi[3];
+};
+
+// Initialisation.
+void launch_init_nodes(const DomView &d, const double origin[3], const double extent[3],
+                       cudaStream_t s);
+// kind: 0 Sedov (rho0, e0, E), 1 USER (rho in d.P scratch, e already in place),
+// 2 USER_MASS (m already in place, e already in place).
+void launch_init_zones(const DomView &d, int kind, double rho0, double e0, double E,
+                       cudaStream_t s);
+// dt^0 (S2-S6 at x^0 with no predictor) over owned zones -> st->dtz_acc, error flags.
+void launch_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+void launch_finalize_init(DevState *st, double dt_first, double dt_init, double dt_max,
+                          double t_stop, double t0, cudaStream_t s);
+
+// Split 3-kernel pipeline (naive, obviously-correct path; HYDRO_FLAG_SPLIT).
+void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+void launch_node_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+void launch_energy_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+
+// Fused single-kernel cycle (default path).
+void launch_cycle_fused(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+
+// End of cycle: S9 dt / time update and error latch.
+void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s);
+
+// Intra-GPU ghost exchange of the next-parity state over a table of slab copies.
+void launch_halo_copy(const DomView *views_dev, const HaloCopy *pairs_dev, int npairs,
+                      cudaStream_t s);
+
+// get_fields: derived zone fields (rho, p, q, c, vol) at (x, u) with no predictor into d.aux.
+void launch_derive(const DomView &d, const Phys &ph, cudaStream_t s);
+
+}  // namespace hydro

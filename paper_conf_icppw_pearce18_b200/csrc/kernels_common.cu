@@ -1,0 +1,349 @@
+// kernels_common.cu -- initialisation, dt bookkeeping (S9), halo copy and output derivation
+// kernels, plus the split 3-kernel pipeline (zone / node / energy) that serves as the plain,
+// one-thread-per-element GPU path (HYDRO_FLAG_SPLIT).  The fused default path is in
+// kernel_fused.cu.
+#include <cmath>
+
+#include "kernels.h"
+#include "zone_physics.cuh"
+
+namespace hydro {
+
+namespace {
+
+constexpr int BX = 32, BY = 4;
+
+__device__ __forceinline__ bool stopped(const DevState *st) {
+  return (st->halted | st->done) != 0u;
+}
+
+__device__ __forceinline__ bool exists_zone(const DomView &d, int i, int j, int k) {
+  const int64_t gx = d.lo[0] + i, gy = d.lo[1] + j, gz = d.lo[2] + k;
+  return gx >= 0 && gx < d.N[0] && gy >= 0 && gy < d.N[1] && gz >= 0 && gz < d.N[2];
+}
+
+__device__ __forceinline__ int64_t global_zone(const DomView &d, int i, int j, int k) {
+  return ((d.lo[2] + k) * (int64_t)d.N[1] + (d.lo[1] + j)) * (int64_t)d.N[0] + (d.lo[0] + i);
+}
+
+// Gather the 8 corners of local zone (i,j,k): positions advanced by hh*u, and velocities.
+__device__ __forceinline__ void gather(const DomView &d, int i, int j, int k, double hh,
+                                       double X[8], double Y[8], double Z[8], double U[8],
+                                       double V[8], double W[8]) {
+#pragma unroll
+  for (int l = 0; l < 8; ++l) {
+    const int64_t id = d.nid(i + (l & 1), j + ((l >> 1) & 1), k + ((l >> 2) & 1));
+    U[l] = d.u[id];
+    V[l] = d.v[id];
+    W[l] = d.w[id];
+    X[l] = d.x[id] + hh * U[l];
+    Y[l] = d.y[id] + hh * V[l];
+    Z[l] = d.z[id] + hh * W[l];
+  }
+}
+
+__device__ __forceinline__ void flag_error(DevState *st, unsigned bits, int64_t gzone) {
+  atomicOr(&st->err, bits);
+  atomicMin(&st->bad_zone, (unsigned long long)gzone);
+}
+
+// ------------------------------------------------------------------------------- init
+__global__ void k_init_nodes(DomView d, double ox, double oy, double oz, double lx, double ly,
+                             double lz) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x - 1;
+  const int j = blockIdx.y * blockDim.y + threadIdx.y - 1;
+  const int k = blockIdx.z - 1;
+  if (i > d.n[0] + 1 || j > d.n[1] + 1) return;
+  const int64_t id = d.nid(i, j, k);
+  // reading R1: origin + (extent*g)/N (also for ghost nodes beyond the physical boundary)
+  const double X = ox + (lx * (double)(d.lo[0] + i)) / (double)d.N[0];
+  const double Y = oy + (ly * (double)(d.lo[1] + j)) / (double)d.N[1];
+  const double Z = oz + (lz * (double)(d.lo[2] + k)) / (double)d.N[2];
+  const_cast<double *>(d.x)[id] = X;
+  const_cast<double *>(d.y)[id] = Y;
+  const_cast<double *>(d.z)[id] = Z;
+  d.xn[id] = X;
+  d.yn[id] = Y;
+  d.zn[id] = Z;
+}
+
+__global__ void k_init_zones(DomView d, int kind, double rho0, double e0, double E) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x - 1;
+  const int j = blockIdx.y * blockDim.y + threadIdx.y - 1;
+  const int k = blockIdx.z - 1;
+  if (i > d.n[0] || j > d.n[1] || !exists_zone(d, i, j, k)) return;
+  double X[8], Y[8], Z[8], U[8], Vv[8], W[8], Bx[8], By[8], Bz[8], V, A2;
+  gather(d, i, j, k, 0.0, X, Y, Z, U, Vv, W);
+  hex_geometry(X, Y, Z, Bx, By, Bz, V, A2);
+  const int64_t id = d.zid(i, j, k);
+  double *m = const_cast<double *>(d.m);
+  double *e = const_cast<double *>(d.e);
+  if (kind == 0) {
+    m[id] = rho0 * V;
+    const bool corner = d.lo[0] + i == 0 && d.lo[1] + j == 0 && d.lo[2] + k == 0;
+    e[id] = corner ? E / m[id] : e0;
+  } else if (kind == 1) {
+    m[id] = d.P[id] * V;  // USER: rho staged in the P scratch
+  }
+}
+
+// dt^0: S2-S6 at x^0 with no predictor over owned zones.
+__global__ void k_dt0(DomView d, Phys ph, DevState *st) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int j = blockIdx.y * blockDim.y + threadIdx.y;
+  const int k = blockIdx.z;
+  double dtz = INFINITY;
+  if (i < d.n[0] && j < d.n[1]) {
+    double X[8], Y[8], Z[8], U[8], Vv[8], W[8], Bx[8], By[8], Bz[8], V, A2;
+    gather(d, i, j, k, 0.0, X, Y, Z, U, Vv, W);
+    hex_geometry(X, Y, Z, Bx, By, Bz, V, A2);
+    double DV = 0.0;
+#pragma unroll
+    for (int l = 0; l < 8; ++l) DV += U[l] * Bx[l] + Vv[l] * By[l] + W[l] * Bz[l];
+    const int64_t id = d.zid(i, j, k);
+    const ZoneEos r = zone_eos(V, A2, DV, d.m[id], d.e[id], 0.0, ph);
+    if (!(V > 0.0)) flag_error(st, ERR_TANGLED, global_zone(d, i, j, k));
+    dtz = (r.dtz == r.dtz) ? r.dtz : INFINITY;
+  }
+  block_min_dt(dtz, &st->dtz_acc);
+}
+
+__global__ void k_finalize_init(DevState *st, double dt_first, double dt_init, double dt_max,
+                                double t_stop, double t0) {
+  const double dtmin = __longlong_as_double((long long)st->dtz_acc);
+  double dt = dt_first > 0.0 ? dt_first : fmin(fmin(dt_init, dt_max), dtmin);
+  if (t_stop > 0.0) dt = fmin(dt, t_stop - t0);
+  st->t = t0;
+  st->dt = dt;
+  st->dtz_last = dtmin;
+  st->dtz_acc = (unsigned long long)__double_as_longlong(INFINITY);
+  st->cycle = 0;
+  st->halted = st->err;
+  st->done = (t_stop > 0.0 && t0 >= t_stop) ? 1u : 0u;
+}
+
+// S9: t' = t + dt, dt' = min(min(growth*dt, dt_max), min_z dt_z), t_stop clamp;
+// latch the cycle's error bits so later cycles become no-ops (the state stays the one after the
+// failing cycle, as in the oracle).
+__global__ void k_finalize(DevState *st, Phys ph) {
+  if (st->halted | st->done) return;
+  const double dtmin = __longlong_as_double((long long)st->dtz_acc);
+  const double dt = st->dt;
+  const double tn = st->t + dt;
+  double dtn = fmin(fmin(ph.dt_growth * dt, ph.dt_max), dtmin);
+  const bool stop = ph.t_stop > 0.0 && tn >= ph.t_stop;
+  if (ph.t_stop > 0.0) dtn = fmin(dtn, ph.t_stop - tn);
+  st->t = tn;
+  st->dt = dtn;
+  st->dtz_last = dtmin;
+  st->cycle += 1;
+  st->dtz_acc = (unsigned long long)__double_as_longlong(INFINITY);
+  unsigned err = st->err;
+  if (!(isfinite(dtn) && dtn > 0.0) && !stop) err |= ERR_NONFINITE;
+  st->halted = err;
+  st->done = stop ? 1u : 0u;
+}
+
+// ------------------------------------------------------------------ split pipeline
+// K1: S1-S6 for every existing local zone (owned and ghost): P and the 24 corner-vector
+// components to scratch, dt_z min over owned zones.
+__global__ void k_zone_split(DomView d, Phys ph, DevState *st) {
+  if (stopped(st)) return;
+  const int i = blockIdx.x * blockDim.x + threadIdx.x - 1;
+  const int j = blockIdx.y * blockDim.y + threadIdx.y - 1;
+  const int k = blockIdx.z - 1;
+  const double hh = 0.5 * st->dt;
+  double dtz = INFINITY;
+  if (i <= d.n[0] && j <= d.n[1] && exists_zone(d, i, j, k)) {
+    double X[8], Y[8], Z[8], U[8], Vv[8], W[8], Bx[8], By[8], Bz[8], V, A2;
+    gather(d, i, j, k, hh, X, Y, Z, U, Vv, W);
+    hex_geometry(X, Y, Z, Bx, By, Bz, V, A2);
+    double DV = 0.0;
+#pragma unroll
+    for (int l = 0; l < 8; ++l) DV += U[l] * Bx[l] + Vv[l] * By[l] + W[l] * Bz[l];
+    const int64_t id = d.zid(i, j, k);
+    const ZoneEos r = zone_eos(V, A2, DV, d.m[id], d.e[id], hh, ph);
+    d.P[id] = r.P;
+#pragma unroll
+    for (int l = 0; l < 8; ++l) {
+      d.B[(3 * l + 0) * d.nzone + id] = Bx[l];
+      d.B[(3 * l + 1) * d.nzone + id] = By[l];
+      d.B[(3 * l + 2) * d.nzone + id] = Bz[l];
+    }
+    const bool owned = i >= 0 && j >= 0 && k >= 0 && i < d.n[0] && j < d.n[1] && k < d.n[2];
+    if (owned) {
+      if (!(V > 0.0)) flag_error(st, ERR_TANGLED, global_zone(d, i, j, k));
+      else if (!isfinite(r.P)) flag_error(st, ERR_NONFINITE, global_zone(d, i, j, k));
+      dtz = (r.dtz == r.dtz) ? r.dtz : INFINITY;
+    }
+  }
+  block_min_dt(dtz, &st->dtz_acc);
+}
+
+// K2: S5 + S7 for owned nodes: gather f = P*B from the existing zones around the node,
+// acceleration, reflecting walls, velocity and position update.
+__global__ void k_node_split(DomView d, Phys ph, DevState *st) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int j = blockIdx.y * blockDim.y + threadIdx.y;
+  const int k = blockIdx.z;
+  if (i > d.n[0] || j > d.n[1]) return;
+  const int64_t id = d.nid(i, j, k);
+  if (stopped(st)) {
+    d.xn[id] = d.x[id]; d.yn[id] = d.y[id]; d.zn[id] = d.z[id];
+    d.un[id] = d.u[id]; d.vn[id] = d.v[id]; d.wn[id] = d.w[id];
+    return;
+  }
+  const double dt = st->dt;
+  double Fx = 0.0, Fy = 0.0, Fz = 0.0, ms = 0.0;
+#pragma unroll
+  for (int lp = 0; lp < 8; ++lp) {
+    const int zi = i - 1 + (lp & 1), zj = j - 1 + ((lp >> 1) & 1), zk = k - 1 + ((lp >> 2) & 1);
+    if (!exists_zone(d, zi, zj, zk)) continue;
+    const int64_t z = d.zid(zi, zj, zk);
+    const int l = 7 - lp;
+    const double P = d.P[z];
+    Fx += P * d.B[(3 * l + 0) * d.nzone + z];
+    Fy += P * d.B[(3 * l + 1) * d.nzone + z];
+    Fz += P * d.B[(3 * l + 2) * d.nzone + z];
+    ms += d.m[z];
+  }
+  const double rinv = 1.0 / (0.125 * ms);
+  double ax = Fx * rinv, ay = Fy * rinv, az = Fz * rinv;
+  const int64_t g[3] = {d.lo[0] + i, d.lo[1] + j, d.lo[2] + k};
+  const uint32_t rm = ph.reflect_mask;
+  if ((g[0] == 0 && (rm & 1u)) || (g[0] == d.N[0] && (rm & 2u))) ax = 0.0;
+  if ((g[1] == 0 && (rm & 4u)) || (g[1] == d.N[1] && (rm & 8u))) ay = 0.0;
+  if ((g[2] == 0 && (rm & 16u)) || (g[2] == d.N[2] && (rm & 32u))) az = 0.0;
+  const double u = d.u[id], v = d.v[id], w = d.w[id];
+  const double un = u + dt * ax, vn = v + dt * ay, wn = w + dt * az;
+  const double uh = (u + un) * 0.5, vh = (v + vn) * 0.5, wh = (w + wn) * 0.5;
+  d.un[id] = un;
+  d.vn[id] = vn;
+  d.wn[id] = wn;
+  d.xn[id] = d.x[id] + dt * uh;
+  d.yn[id] = d.y[id] + dt * vh;
+  d.zn[id] = d.z[id] + dt * wh;
+}
+
+// K3: S8 for owned zones: W = sum_l (P B_l).u_half_l, e' = e - dt W / m.
+__global__ void k_energy_split(DomView d, Phys ph, DevState *st) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int j = blockIdx.y * blockDim.y + threadIdx.y;
+  const int k = blockIdx.z;
+  if (i >= d.n[0] || j >= d.n[1]) return;
+  const int64_t id = d.zid(i, j, k);
+  if (stopped(st)) {
+    d.en[id] = d.e[id];
+    return;
+  }
+  const double dt = st->dt;
+  const double P = d.P[id];
+  double Wk = 0.0;
+#pragma unroll
+  for (int l = 0; l < 8; ++l) {
+    const int64_t n = d.nid(i + (l & 1), j + ((l >> 1) & 1), k + ((l >> 2) & 1));
+    const double uh = (d.u[n] + d.un[n]) * 0.5;
+    const double vh = (d.v[n] + d.vn[n]) * 0.5;
+    const double wh = (d.w[n] + d.wn[n]) * 0.5;
+    Wk += (P * d.B[(3 * l + 0) * d.nzone + id]) * uh + (P * d.B[(3 * l + 1) * d.nzone + id]) * vh +
+          (P * d.B[(3 * l + 2) * d.nzone + id]) * wh;
+  }
+  d.en[id] = d.e[id] - dt * Wk / d.m[id];
+}
+
+// ---------------------------------------------------------------------- halo copy
+__global__ void k_halo_copy(const DomView *views, const HaloCopy *pairs) {
+  const HaloCopy p = pairs[blockIdx.y];
+  const DomView &D = views[p.dst];
+  const DomView &S = views[p.src];
+  const int64_t nx = p.nhi[0] - p.nlo[0], ny = p.nhi[1] - p.nlo[1], nz = p.nhi[2] - p.nlo[2];
+  const int64_t nn = nx * ny * nz;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nn;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = t % nx, b = (t / nx) % ny, c = t / (nx * ny);
+    const int64_t gx = p.nlo[0] + a, gy = p.nlo[1] + b, gz = p.nlo[2] + c;
+    const int64_t di = D.nid((int)(gx - D.lo[0]), (int)(gy - D.lo[1]), (int)(gz - D.lo[2]));
+    const int64_t si = S.nid((int)(gx - S.lo[0]), (int)(gy - S.lo[1]), (int)(gz - S.lo[2]));
+    D.xn[di] = S.xn[si];
+    D.yn[di] = S.yn[si];
+    D.zn[di] = S.zn[si];
+    D.un[di] = S.un[si];
+    D.vn[di] = S.vn[si];
+    D.wn[di] = S.wn[si];
+  }
+  const int64_t zx = p.zhi[0] - p.zlo[0], zy = p.zhi[1] - p.zlo[1], zz = p.zhi[2] - p.zlo[2];
+  const int64_t nzn = zx * zy * zz;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nzn;
+       t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = t % zx, b = (t / zx) % zy, c = t / (zx * zy);
+    const int64_t gx = p.zlo[0] + a, gy = p.zlo[1] + b, gz = p.zlo[2] + c;
+    D.en[D.zid((int)(gx - D.lo[0]), (int)(gy - D.lo[1]), (int)(gz - D.lo[2]))] =
+        S.en[S.zid((int)(gx - S.lo[0]), (int)(gy - S.lo[1]), (int)(gz - S.lo[2]))];
+  }
+}
+
+// ------------------------------------------------------------------------ outputs
+__global__ void k_derive(DomView d, Phys ph) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int j = blockIdx.y * blockDim.y + threadIdx.y;
+  const int k = blockIdx.z;
+  if (i >= d.n[0] || j >= d.n[1]) return;
+  double X[8], Y[8], Z[8], U[8], Vv[8], W[8], Bx[8], By[8], Bz[8], V, A2;
+  gather(d, i, j, k, 0.0, X, Y, Z, U, Vv, W);
+  hex_geometry(X, Y, Z, Bx, By, Bz, V, A2);
+  double DV = 0.0;
+#pragma unroll
+  for (int l = 0; l < 8; ++l) DV += U[l] * Bx[l] + Vv[l] * By[l] + W[l] * Bz[l];
+  const int64_t id = d.zid(i, j, k);
+  const ZoneEos r = zone_eos(V, A2, DV, d.m[id], d.e[id], 0.0, ph);
+  d.aux[0 * d.nzone + id] = r.rho;
+  d.aux[1 * d.nzone + id] = r.p;
+  d.aux[2 * d.nzone + id] = r.q;
+  d.aux[3 * d.nzone + id] = r.c;
+  d.aux[4 * d.nzone + id] = V;
+}
+
+dim3 grid_for(int nx, int ny, int nz) {
+  return dim3((nx + BX - 1) / BX, (ny + BY - 1) / BY, nz);
+}
+
+}  // namespace
+
+void launch_init_nodes(const DomView &d, const double o[3], const double L[3], cudaStream_t s) {
+  k_init_nodes<<<grid_for(d.n[0] + 3, d.n[1] + 3, d.n[2] + 3), dim3(BX, BY), 0, s>>>(
+      d, o[0], o[1], o[2], L[0], L[1], L[2]);
+}
+void launch_init_zones(const DomView &d, int kind, double rho0, double e0, double E,
+                       cudaStream_t s) {
+  k_init_zones<<<grid_for(d.n[0] + 2, d.n[1] + 2, d.n[2] + 2), dim3(BX, BY), 0, s>>>(
+      d, kind, rho0, e0, E);
+}
+void launch_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
+  k_dt0<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph, st);
+}
+void launch_finalize_init(DevState *st, double dt_first, double dt_init, double dt_max,
+                          double t_stop, double t0, cudaStream_t s) {
+  k_finalize_init<<<1, 1, 0, s>>>(st, dt_first, dt_init, dt_max, t_stop, t0);
+}
+void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
+  k_zone_split<<<grid_for(d.n[0] + 2, d.n[1] + 2, d.n[2] + 2), dim3(BX, BY), 0, s>>>(d, ph, st);
+}
+void launch_node_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
+  k_node_split<<<grid_for(d.n[0] + 1, d.n[1] + 1, d.n[2] + 1), dim3(BX, BY), 0, s>>>(d, ph, st);
+}
+void launch_energy_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
+  k_energy_split<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph, st);
+}
+void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s) {
+  k_finalize<<<1, 1, 0, s>>>(st, ph);
+}
+void launch_halo_copy(const DomView *views_dev, const HaloCopy *pairs_dev, int npairs,
+                      cudaStream_t s) {
+  if (npairs <= 0) return;
+  k_halo_copy<<<dim3(16, npairs), 256, 0, s>>>(views_dev, pairs_dev);
+}
+void launch_derive(const DomView &d, const Phys &ph, cudaStream_t s) {
+  k_derive<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph);
+}
+
+}  // namespace hydro

@@ -1,0 +1,598 @@
+// runtime.cu -- the C ABI of include/hydro.h: context, per-domain device allocation, CUDA-graph
+// capture of a cycle, host<->device field transfer.  One process drives one GPU; all domains
+// assigned to this rank live in its HBM (each rank owns its domains).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <limits>
+#include <string>
+#include <vector>
+
+#include "../../include/hydro.h"
+#include "comm.h"
+#include "kernels.h"
+#include "layout.h"
+
+using namespace hydro;
+
+namespace {
+
+thread_local std::string g_err;
+
+struct LocalDom {
+  int32_t dom;  // global domain index
+  DomainBox box;
+  void *mem = nullptr;
+  size_t bytes = 0;
+  DomView view[2];  // parity p reads view[p].x and writes view[p].xn
+};
+
+}  // namespace
+
+struct hydro_ctx {
+  hydro_config cfg;
+  Layout L;
+  Phys ph;
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  std::vector<LocalDom> doms;
+  std::vector<int32_t> slot_of_dom;  // global domain -> local slot or -1
+  DevState *st = nullptr;
+  DomView *views_dev[2] = {nullptr, nullptr};
+  HaloCopy *local_pairs_dev = nullptr;
+  int n_local_pairs = 0;
+  cudaGraphExec_t graph[2] = {nullptr, nullptr};
+  int parity = 0;
+  bool split = false;
+  bool use_graph = true;
+  int failed = 0;
+  Comm *comm = nullptr;
+  std::string err;
+};
+
+namespace {
+
+int set_err(hydro_ctx *h, int code, const std::string &msg) {
+  g_err = msg;
+  if (h) h->err = msg;
+  return code;
+}
+
+#define CK(call)                                                                       \
+  do {                                                                                 \
+    cudaError_t e_ = (call);                                                           \
+    if (e_ != cudaSuccess)                                                             \
+      return set_err(h, HYDRO_ECUDA, std::string(#call ": ") + cudaGetErrorString(e_)); \
+  } while (0)
+
+size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
+  const int64_t n0 = D.box.n[0], n1 = D.box.n[1], n2 = D.box.n[2];
+  const int64_t nsx = n0 + 3, nsxy = nsx * (n1 + 3), nnode = nsxy * (n2 + 3);
+  const int64_t zsx = n0 + 2, zsxy = zsx * (n1 + 2), nzone = zsxy * (n2 + 2);
+  const size_t nb = align_up(nnode * sizeof(double), 256), zb = align_up(nzone * sizeof(double), 256);
+  // 12 node arrays (2 parities x 6), e x2, m, P, aux x5, optional B x24
+  size_t bytes = 12 * nb + 9 * zb + (split ? 24 * zb : 0);
+  CK(cudaMalloc(&D.mem, bytes));
+  CK(cudaMemsetAsync(D.mem, 0, bytes, h->stream));
+  D.bytes = bytes;
+  char *p = (char *)D.mem;
+  double *nodes[12];
+  for (int a = 0; a < 12; ++a, p += nb) nodes[a] = (double *)p;
+  double *e0 = (double *)p; p += zb;
+  double *e1 = (double *)p; p += zb;
+  double *m = (double *)p; p += zb;
+  double *P = (double *)p; p += zb;
+  double *aux = (double *)p; p += 5 * zb;
+  double *B = split ? (double *)p : nullptr;
+  for (int par = 0; par < 2; ++par) {
+    DomView &v = D.view[par];
+    std::memset(&v, 0, sizeof(v));
+    for (int a = 0; a < 3; ++a) {
+      v.lo[a] = D.box.lo[a];
+      v.n[a] = (int32_t)D.box.n[a];
+      v.N[a] = (int32_t)h->L.N[a];
+    }
+    v.nsx = nsx; v.nsxy = nsxy; v.zsx = zsx; v.zsxy = zsxy;
+    v.nnode = nnode; v.nzone = zb / sizeof(double);  // zone array stride (aux/B planes)
+    double **cur = nodes + 6 * par, **nxt = nodes + 6 * (1 - par);
+    v.x = cur[0]; v.y = cur[1]; v.z = cur[2]; v.u = cur[3]; v.v = cur[4]; v.w = cur[5];
+    v.xn = nxt[0]; v.yn = nxt[1]; v.zn = nxt[2]; v.un = nxt[3]; v.vn = nxt[4]; v.wn = nxt[5];
+    v.e = par ? e1 : e0;
+    v.en = par ? e0 : e1;
+    v.m = m; v.P = P; v.B = B; v.aux = aux;
+    v.dom = D.dom;
+  }
+  return HYDRO_OK;
+}
+
+// Copy a global box between a dense host array (dims gdims, x fastest) and a domain's local
+// array (local index of global g is g - lo + 1 along each axis).
+int copy_box(hydro_ctx *h, bool to_device, double *host, const int64_t gdims[3],
+             const int64_t glo[3], const int64_t ext[3], double *dev, int64_t dsx, int64_t dsy,
+             const int64_t dlo_local[3], cudaStream_t s) {
+  if (ext[0] <= 0 || ext[1] <= 0 || ext[2] <= 0) return HYDRO_OK;
+  cudaMemcpy3DParms p;
+  std::memset(&p, 0, sizeof(p));
+  cudaPitchedPtr hp = make_cudaPitchedPtr(host, gdims[0] * sizeof(double), gdims[0], gdims[1]);
+  cudaPitchedPtr dp = make_cudaPitchedPtr(dev, dsx * sizeof(double), dsx, dsy);
+  cudaPos hpos = make_cudaPos(glo[0] * sizeof(double), glo[1], glo[2]);
+  cudaPos dpos = make_cudaPos(dlo_local[0] * sizeof(double), dlo_local[1], dlo_local[2]);
+  p.extent = make_cudaExtent(ext[0] * sizeof(double), ext[1], ext[2]);
+  if (to_device) {
+    p.srcPtr = hp; p.srcPos = hpos; p.dstPtr = dp; p.dstPos = dpos;
+    p.kind = cudaMemcpyHostToDevice;
+  } else {
+    p.srcPtr = dp; p.srcPos = dpos; p.dstPtr = hp; p.dstPos = hpos;
+    p.kind = cudaMemcpyDeviceToHost;
+  }
+  CK(cudaMemcpy3DAsync(&p, s));
+  return HYDRO_OK;
+}
+
+// Upload global host arrays into every local domain's parity-p arrays (existing owned+ghost
+// entries).  nodes6 may be NULL; zone arrays: e -> e, z6 (rho or mass) -> P scratch or m.
+int upload_state(hydro_ctx *h, int par, const double *const *nodes6, const double *e,
+                 const double *zone_extra, bool extra_is_mass) {
+  const int64_t gn[3] = {h->L.N[0] + 1, h->L.N[1] + 1, h->L.N[2] + 1};
+  const int64_t gz[3] = {h->L.N[0], h->L.N[1], h->L.N[2]};
+  for (LocalDom &D : h->doms) {
+    DomView &v = D.view[par];
+    int64_t nlo[3], next[3], nloc[3], zlo[3], zext[3], zloc[3];
+    for (int a = 0; a < 3; ++a) {
+      const int64_t lo = std::max<int64_t>(D.box.lo[a] - 1, 0);
+      const int64_t hi = std::min<int64_t>(D.box.lo[a] + D.box.n[a] + 1, h->L.N[a]);  // nodes
+      nlo[a] = lo; next[a] = hi - lo + 1; nloc[a] = lo - D.box.lo[a] + 1;
+      const int64_t zl = std::max<int64_t>(D.box.lo[a] - 1, 0);
+      const int64_t zh = std::min<int64_t>(D.box.lo[a] + D.box.n[a] + 1, h->L.N[a]);  // excl
+      zlo[a] = zl; zext[a] = zh - zl; zloc[a] = zl - D.box.lo[a] + 1;
+    }
+    if (nodes6) {
+      double *dst[6] = {const_cast<double *>(v.x), const_cast<double *>(v.y),
+                        const_cast<double *>(v.z), const_cast<double *>(v.u),
+                        const_cast<double *>(v.v), const_cast<double *>(v.w)};
+      for (int f = 0; f < 6; ++f) {
+        int rc = copy_box(h, true, const_cast<double *>(nodes6[f]), gn, nlo, next, dst[f], v.nsx,
+                          v.nsxy / v.nsx, nloc, h->stream);
+        if (rc) return rc;
+      }
+    }
+    if (e) {
+      int rc = copy_box(h, true, const_cast<double *>(e), gz, zlo, zext,
+                        const_cast<double *>(v.e), v.zsx, v.zsxy / v.zsx, zloc, h->stream);
+      if (rc) return rc;
+    }
+    if (zone_extra) {
+      double *dst = extra_is_mass ? const_cast<double *>(v.m) : v.P;
+      int rc = copy_box(h, true, const_cast<double *>(zone_extra), gz, zlo, zext, dst, v.zsx,
+                        v.zsxy / v.zsx, zloc, h->stream);
+      if (rc) return rc;
+    }
+  }
+  return HYDRO_OK;
+}
+
+// Enqueue one cycle on stream s reading parity `par`.
+int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
+  for (LocalDom &D : h->doms) {
+    if (h->split) {
+      launch_zone_split(D.view[par], h->ph, h->st, s);
+    }
+  }
+  if (h->split) {
+    if (h->comm) {
+      int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
+      if (rc) return set_err(h, rc, "dt allreduce failed");
+    }
+    for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
+    for (LocalDom &D : h->doms) launch_energy_split(D.view[par], h->ph, h->st, s);
+  } else {
+    for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], h->ph, h->st, s);
+    if (h->comm) {
+      int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
+      if (rc) return set_err(h, rc, "dt allreduce failed");
+    }
+  }
+  launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
+  if (h->comm) {
+    int rc = comm_halo(h->comm, par, s);
+    if (rc) return set_err(h, rc, "halo exchange failed");
+  }
+  launch_finalize(h->st, h->ph, s);
+  CK(cudaGetLastError());
+  return HYDRO_OK;
+}
+
+int build_graphs(hydro_ctx *h) {
+  for (int par = 0; par < 2; ++par) {
+    cudaGraph_t g;
+    CK(cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal));
+    int rc = enqueue_cycle(h, par, h->stream);
+    cudaError_t e = cudaStreamEndCapture(h->stream, &g);
+    if (rc) return rc;
+    if (e != cudaSuccess) return set_err(h, HYDRO_ECUDA, cudaGetErrorString(e));
+    CK(cudaGraphInstantiate(&h->graph[par], g, 0));
+    CK(cudaGraphDestroy(g));
+  }
+  return HYDRO_OK;
+}
+
+int read_info(hydro_ctx *h, hydro_info *info, cudaStream_t s) {
+  DevState st;
+  CK(cudaMemcpyAsync(&st, h->st, sizeof(st), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  int status = HYDRO_OK;
+  if (st.halted & ERR_TANGLED) status = HYDRO_ETANGLED;
+  else if (st.halted & ERR_NONFINITE) status = HYDRO_ENONFINITE;
+  if (h->comm) status = comm_status_agree(h->comm, status);
+  if (info) {
+    info->t = st.t;
+    info->dt = st.dt;
+    info->cycle = (int64_t)st.cycle;
+    info->dt_min_zone = st.dtz_last;
+    info->status = status;
+    info->bad_zone = (st.bad_zone == ~0ull) ? -1 : (int64_t)st.bad_zone;
+  }
+  return status;
+}
+
+bool valid_phys(const hydro_config *c) {
+  return c->gamma > 1.0 && c->q_lin >= 0.0 && c->q_quad >= 0.0 && c->cfl > 0.0 &&
+         c->c_vol > 0.0 && c->dt_growth > 0.0 && c->dt_max > 0.0 &&
+         std::isfinite(c->origin[0]) && c->extent[0] > 0.0 && c->extent[1] > 0.0 &&
+         c->extent[2] > 0.0;
+}
+
+}  // namespace
+
+extern "C" {
+
+int hydro_abi_version(void) { return HYDRO_ABI_VERSION; }
+
+void hydro_config_default(hydro_config *c) {
+  std::memset(c, 0, sizeof(*c));
+  c->abi_version = HYDRO_ABI_VERSION;
+  for (int a = 0; a < 3; ++a) {
+    c->n[a] = 32;
+    c->origin[a] = 0.0;
+    c->extent[a] = 1.2;
+    c->ndom[a] = 1;
+  }
+  c->gamma = 1.4;
+  c->q_lin = 0.5;
+  c->q_quad = 2.0;
+  c->cfl = 0.3;
+  c->c_vol = 0.1;
+  c->dt_growth = 1.1;
+  c->dt_max = INFINITY;
+  c->dt_init = INFINITY;
+  c->reflect_mask = 0x3f;
+  c->init_kind = HYDRO_INIT_SEDOV;
+  c->rho0 = 1.0;
+  c->sedov_energy = 0.851072 / 8.0;
+  c->nranks = 1;
+}
+
+const char *hydro_strerror(int s) {
+  switch (s) {
+    case HYDRO_OK: return "ok";
+    case HYDRO_EINVAL: return "invalid argument";
+    case HYDRO_ENOMEM: return "out of memory";
+    case HYDRO_ECUDA: return "CUDA error";
+    case HYDRO_ENCCL: return "communicator error";
+    case HYDRO_ETANGLED: return "tangled mesh (zone volume <= 0)";
+    case HYDRO_ENONFINITE: return "non-finite pressure or dt";
+    case HYDRO_EDTMIN: return "dt below floor";
+    case HYDRO_ESTATE: return "context in failed state";
+    default: return "unknown status";
+  }
+}
+
+const char *hydro_last_error(const hydro_ctx *h) { return h ? h->err.c_str() : g_err.c_str(); }
+
+int hydro_comm_unique_id(void *out128) { return comm_unique_id(out128); }
+
+int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
+  hydro_ctx *h = nullptr;
+  if (!cfg || !out) return set_err(nullptr, HYDRO_EINVAL, "NULL argument");
+  *out = nullptr;
+  if (cfg->abi_version != HYDRO_ABI_VERSION)
+    return set_err(nullptr, HYDRO_EINVAL, "abi_version mismatch");
+  if (!valid_phys(cfg)) return set_err(nullptr, HYDRO_EINVAL, "invalid physics parameters");
+  if (cfg->init_kind < 0 || cfg->init_kind > 2)
+    return set_err(nullptr, HYDRO_EINVAL, "invalid init_kind");
+  if (cfg->init_kind != HYDRO_INIT_SEDOV)
+    for (int f = 0; f < 8; ++f)
+      if (!cfg->user[f]) return set_err(nullptr, HYDRO_EINVAL, "USER init needs 8 arrays");
+  h = new hydro_ctx();
+  h->cfg = *cfg;
+  std::memset(h->cfg.user, 0, sizeof(h->cfg.user));
+  for (int a = 0; a < 3; ++a) h->cfg.cuts[a] = nullptr;
+  h->cfg.dom_to_rank = nullptr;
+  h->cfg.rank_weight = nullptr;
+  h->cfg.comm_id = nullptr;
+  std::string err;
+  int rc = layout_build(cfg, &h->L, &err);
+  if (rc) {
+    delete h;
+    return set_err(nullptr, rc, err);
+  }
+  h->ph.gamma = cfg->gamma;
+  h->ph.gm1 = cfg->gamma - 1.0;
+  h->ph.ggm1 = cfg->gamma * (cfg->gamma - 1.0);
+  h->ph.q_lin = cfg->q_lin;
+  h->ph.q_quad = cfg->q_quad;
+  h->ph.cfl = cfg->cfl;
+  h->ph.c_vol = cfg->c_vol;
+  h->ph.dt_growth = cfg->dt_growth;
+  h->ph.dt_max = cfg->dt_max;
+  h->ph.t_stop = cfg->t_stop;
+  h->ph.reflect_mask = cfg->reflect_mask;
+  h->split = true;  // TEMP: fused kernel not yet in tree
+  h->use_graph = (cfg->flags & HYDRO_FLAG_NO_GRAPH) == 0;
+  h->device = cfg->device;
+  *out = nullptr;
+  auto fail = [&](int code) {
+    hydro_destroy(h);
+    return code;
+  };
+  {
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0) {
+      set_err(h, HYDRO_ECUDA, "no CUDA device available (the library has no CPU path)");
+      return fail(HYDRO_ECUDA);
+    }
+  }
+  if (cudaSetDevice(h->device) != cudaSuccess) {
+    set_err(h, HYDRO_ECUDA, "cudaSetDevice failed");
+    return fail(HYDRO_ECUDA);
+  }
+  if ((rc = [&]() -> int {
+         CK(cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking));
+         CK(cudaMalloc(&h->st, sizeof(DevState)));
+         DevState s0;
+         std::memset(&s0, 0, sizeof(s0));
+         s0.dtz_acc = (unsigned long long)0x7ff0000000000000ull;  // +inf
+         s0.bad_zone = ~0ull;
+         CK(cudaMemcpyAsync(h->st, &s0, sizeof(s0), cudaMemcpyHostToDevice, h->stream));
+         h->slot_of_dom.assign(h->L.dom.size(), -1);
+         for (size_t d = 0; d < h->L.dom.size(); ++d) {
+           if (h->L.dom[d].rank != cfg->rank) continue;
+           LocalDom D;
+           D.dom = (int32_t)d;
+           D.box = h->L.dom[d];
+           h->slot_of_dom[d] = (int32_t)h->doms.size();
+           h->doms.push_back(D);
+         }
+         for (LocalDom &D : h->doms) {
+           int r = alloc_domain(h, D, h->split);
+           if (r) return r;
+         }
+         // device views and intra-GPU halo pairs
+         for (int par = 0; par < 2; ++par) {
+           CK(cudaMalloc(&h->views_dev[par], sizeof(DomView) * std::max<size_t>(1, h->doms.size())));
+           std::vector<DomView> vv;
+           for (LocalDom &D : h->doms) vv.push_back(D.view[par]);
+           if (!vv.empty())
+             CK(cudaMemcpyAsync(h->views_dev[par], vv.data(), sizeof(DomView) * vv.size(),
+                                cudaMemcpyHostToDevice, h->stream));
+         }
+         std::vector<HaloCopy> lp;
+         std::vector<HaloPair> remote;
+         for (const HaloPair &P : h->L.pairs) {
+           const bool dst_local = h->slot_of_dom[P.dst] >= 0;
+           const bool src_local = h->slot_of_dom[P.src] >= 0;
+           if (dst_local && src_local) {
+             HaloCopy c;
+             c.dst = h->slot_of_dom[P.dst];
+             c.src = h->slot_of_dom[P.src];
+             for (int a = 0; a < 3; ++a) {
+               c.nlo[a] = P.nlo[a]; c.nhi[a] = P.nhi[a]; c.zlo[a] = P.zlo[a]; c.zhi[a] = P.zhi[a];
+             }
+             lp.push_back(c);
+           } else if (dst_local || src_local) {
+             remote.push_back(P);
+           }
+         }
+         h->n_local_pairs = (int)lp.size();
+         if (!lp.empty()) {
+           CK(cudaMalloc(&h->local_pairs_dev, sizeof(HaloCopy) * lp.size()));
+           CK(cudaMemcpyAsync(h->local_pairs_dev, lp.data(), sizeof(HaloCopy) * lp.size(),
+                              cudaMemcpyHostToDevice, h->stream));
+         }
+         if (cfg->nranks > 1) {
+           int r = comm_create(&h->comm, cfg, h->L, remote, h->slot_of_dom, h->doms.empty() ? nullptr : nullptr,
+                               h->stream, &h->err);
+           if (r) return r;
+           std::vector<const DomView *> v0, v1;
+           for (LocalDom &D : h->doms) {
+             v0.push_back(&D.view[0]);
+             v1.push_back(&D.view[1]);
+           }
+           r = comm_bind_views(h->comm, v0.data(), v1.data(), (int)h->doms.size(), &h->err);
+           if (r) return r;
+         }
+         // initial state
+         for (LocalDom &D : h->doms) launch_init_nodes(D.view[0], cfg->origin, cfg->extent, h->stream);
+         if (cfg->init_kind != HYDRO_INIT_SEDOV) {
+           int r = upload_state(h, 0, cfg->user, cfg->user[7], cfg->user[6],
+                                cfg->init_kind == HYDRO_INIT_USER_MASS);
+           if (r) return r;
+         }
+         for (LocalDom &D : h->doms)
+           launch_init_zones(D.view[0], cfg->init_kind, cfg->rho0, cfg->e0, cfg->sedov_energy,
+                             h->stream);
+         for (LocalDom &D : h->doms) launch_dt0(D.view[0], h->ph, h->st, h->stream);
+         if (h->comm) {
+           int r = comm_dt_min(h->comm, &h->st->dtz_acc, h->stream);
+           if (r) return set_err(h, r, "dt allreduce failed");
+         }
+         launch_finalize_init(h->st, cfg->dt_first, cfg->dt_init, cfg->dt_max, cfg->t_stop,
+                              cfg->t0, h->stream);
+         CK(cudaGetLastError());
+         CK(cudaStreamSynchronize(h->stream));
+         return HYDRO_OK;
+       }()) != HYDRO_OK)
+    return fail(rc);
+  hydro_info info;
+  int st = read_info(h, &info, h->stream);
+  if (st == HYDRO_ETANGLED) {
+    set_err(h, st, "initial mesh has a zone with volume <= 0");
+    return fail(st);
+  }
+  if (h->use_graph && (rc = build_graphs(h)) != HYDRO_OK) return fail(rc);
+  *out = h;
+  return HYDRO_OK;
+}
+
+int hydro_step(hydro_ctx *h, int32_t ncycles, void *cuda_stream, hydro_info *info) {
+  if (!h || ncycles < 0) return set_err(h, HYDRO_EINVAL, "bad argument");
+  if (h->failed) return set_err(h, HYDRO_ESTATE, "context failed earlier");
+  CK(cudaSetDevice(h->device));
+  cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : h->stream;
+  for (int32_t c = 0; c < ncycles; ++c) {
+    if (h->use_graph) {
+      CK(cudaGraphLaunch(h->graph[h->parity], s));
+    } else {
+      int rc = enqueue_cycle(h, h->parity, s);
+      if (rc) return rc;
+    }
+    h->parity ^= 1;
+  }
+  const int status = read_info(h, info, s);
+  if (status < 0 && status != HYDRO_ECUDA) h->failed = status;
+  return status;
+}
+
+int hydro_get_info(hydro_ctx *h, hydro_info *info) {
+  if (!h) return HYDRO_EINVAL;
+  CK(cudaSetDevice(h->device));
+  read_info(h, info, h->stream);
+  return HYDRO_OK;
+}
+
+int hydro_get_box(hydro_ctx *h, const int64_t lo[3], const int64_t hi[3], uint32_t mask,
+                  double *const *out) {
+  if (!h || !lo || !hi || !out) return set_err(h, HYDRO_EINVAL, "NULL argument");
+  for (int a = 0; a < 3; ++a)
+    if (lo[a] < 0 || hi[a] > h->L.N[a] || hi[a] <= lo[a])
+      return set_err(h, HYDRO_EINVAL, "box out of range");
+  for (int f = 0; f < HYDRO_NFIELDS; ++f)
+    if ((mask >> f & 1u) && !out[f]) return set_err(h, HYDRO_EINVAL, "missing output array");
+  CK(cudaSetDevice(h->device));
+  const int par = h->parity;
+  const bool derived = (mask & (HYDRO_F_RHO | HYDRO_F_P | HYDRO_F_Q | HYDRO_F_C | HYDRO_F_VOL)) != 0;
+  if (derived)
+    for (LocalDom &D : h->doms) launch_derive(D.view[par], h->ph, h->stream);
+  const int64_t bn[3] = {hi[0] - lo[0] + 1, hi[1] - lo[1] + 1, hi[2] - lo[2] + 1};
+  const int64_t bz[3] = {hi[0] - lo[0], hi[1] - lo[1], hi[2] - lo[2]};
+  for (LocalDom &D : h->doms) {
+    const DomView &v = D.view[par];
+    // nodes written by this domain: lowest-index owner rule per axis
+    int64_t nlo[3], next[3], zlo[3], zext[3];
+    bool any_n = true, any_z = true;
+    for (int a = 0; a < 3; ++a) {
+      const int64_t own_lo = D.box.lo[a] + (D.box.idx[a] > 0 ? 1 : 0);
+      const int64_t own_hi = D.box.lo[a] + D.box.n[a];  // inclusive
+      nlo[a] = std::max(own_lo, lo[a]);
+      next[a] = std::min(own_hi, hi[a]) - nlo[a] + 1;
+      if (next[a] <= 0) any_n = false;
+      zlo[a] = std::max(D.box.lo[a], lo[a]);
+      zext[a] = std::min(D.box.lo[a] + D.box.n[a], hi[a]) - zlo[a];
+      if (zext[a] <= 0) any_z = false;
+    }
+    if (any_n) {
+      const double *src[6] = {v.x, v.y, v.z, v.u, v.v, v.w};
+      int64_t hl[3], dl[3];
+      for (int a = 0; a < 3; ++a) {
+        hl[a] = nlo[a] - lo[a];
+        dl[a] = nlo[a] - D.box.lo[a] + 1;
+      }
+      for (int f = 0; f < 6; ++f) {
+        if (!(mask >> f & 1u)) continue;
+        int rc = copy_box(h, false, out[f], bn, hl, next, const_cast<double *>(src[f]), v.nsx,
+                          v.nsxy / v.nsx, dl, h->stream);
+        if (rc) return rc;
+      }
+    }
+    if (any_z) {
+      int64_t hl[3], dl[3];
+      for (int a = 0; a < 3; ++a) {
+        hl[a] = zlo[a] - lo[a];
+        dl[a] = zlo[a] - D.box.lo[a] + 1;
+      }
+      const double *src[HYDRO_NFIELDS] = {};
+      src[6] = v.aux + 0 * v.nzone;
+      src[7] = v.e;
+      src[8] = v.aux + 1 * v.nzone;
+      src[9] = v.aux + 2 * v.nzone;
+      src[10] = v.aux + 3 * v.nzone;
+      src[11] = v.aux + 4 * v.nzone;
+      src[12] = v.m;
+      for (int f = 6; f < HYDRO_NFIELDS; ++f) {
+        if (!(mask >> f & 1u)) continue;
+        int rc = copy_box(h, false, out[f], bz, hl, zext, const_cast<double *>(src[f]), v.zsx,
+                          v.zsxy / v.zsx, dl, h->stream);
+        if (rc) return rc;
+      }
+    }
+  }
+  CK(cudaStreamSynchronize(h->stream));
+  return HYDRO_OK;
+}
+
+int hydro_get_fields(hydro_ctx *h, uint32_t mask, double *const *out) {
+  if (!h) return set_err(h, HYDRO_EINVAL, "NULL context");
+  const int64_t lo[3] = {0, 0, 0};
+  const int64_t hi[3] = {h->L.N[0], h->L.N[1], h->L.N[2]};
+  return hydro_get_box(h, lo, hi, mask, out);
+}
+
+int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, double t,
+                    double dt) {
+  if (!h || !nodes6 || !e || !(dt > 0.0)) return set_err(h, HYDRO_EINVAL, "bad argument");
+  for (int f = 0; f < 6; ++f)
+    if (!nodes6[f]) return set_err(h, HYDRO_EINVAL, "missing node array");
+  CK(cudaSetDevice(h->device));
+  int rc = upload_state(h, h->parity, nodes6, e, nullptr, false);
+  if (rc) return rc;
+  DevState s0;
+  CK(cudaMemcpyAsync(&s0, h->st, sizeof(s0), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  s0.t = t;
+  s0.dt = dt;
+  s0.err = 0;
+  s0.halted = 0;
+  s0.done = (h->ph.t_stop > 0.0 && t >= h->ph.t_stop) ? 1u : 0u;
+  s0.bad_zone = ~0ull;
+  s0.dtz_acc = (unsigned long long)0x7ff0000000000000ull;
+  CK(cudaMemcpyAsync(h->st, &s0, sizeof(s0), cudaMemcpyHostToDevice, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  h->failed = 0;
+  return HYDRO_OK;
+}
+
+int hydro_destroy(hydro_ctx *h) {
+  if (!h) return HYDRO_OK;
+  cudaSetDevice(h->device);
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  for (int p = 0; p < 2; ++p) {
+    if (h->graph[p]) cudaGraphExecDestroy(h->graph[p]);
+    if (h->views_dev[p]) cudaFree(h->views_dev[p]);
+  }
+  if (h->comm) comm_destroy(h->comm);
+  for (LocalDom &D : h->doms)
+    if (D.mem) cudaFree(D.mem);
+  if (h->local_pairs_dev) cudaFree(h->local_pairs_dev);
+  if (h->st) cudaFree(h->st);
+  if (h->stream) cudaStreamDestroy(h->stream);
+  delete h;
+  return HYDRO_OK;
+}
+
+}  // extern "C"

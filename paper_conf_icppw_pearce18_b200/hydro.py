@@ -1,0 +1,349 @@
+"""Thin Python binding of include/hydro.h (argument marshalling only).
+
+Every step of the cycle runs in the CUDA kernels of ``libhydro_b200.so``; this module only
+fills the C structs, owns host buffers and, for multi-process runs, uses ``torch.distributed``
+to broadcast the communicator id and to combine the per-rank parts of ``fields()``.  There is
+no CPU fallback: if the library or a CUDA device is missing, ``Hydro(...)`` raises.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import math
+import os
+from dataclasses import dataclass
+from typing import Dict, Optional, Sequence
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libhydro_b200.so")
+
+NODE_FIELDS = ("x", "y", "z", "u", "v", "w")
+ZONE_FIELDS = ("rho", "e", "p", "q", "c", "vol", "mass")
+ALL_FIELDS = NODE_FIELDS + ZONE_FIELDS
+ABI_VERSION = 1
+FLAG_NO_GRAPH = 1 << 0
+FLAG_SPLIT = 1 << 1
+
+STATUS = {0: "ok", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENCCL", -5: "ETANGLED",
+          -6: "ENONFINITE", -7: "EDTMIN", -8: "ESTATE"}
+
+
+class HydroConfigC(C.Structure):
+    _fields_ = [
+        ("abi_version", C.c_int32),
+        ("n", C.c_int64 * 3),
+        ("origin", C.c_double * 3),
+        ("extent", C.c_double * 3),
+        ("ndom", C.c_int32 * 3),
+        ("cuts", C.POINTER(C.c_int64) * 3),
+        ("dom_to_rank", C.POINTER(C.c_int32)),
+        ("rank_weight", C.POINTER(C.c_double)),
+        ("gamma", C.c_double), ("q_lin", C.c_double), ("q_quad", C.c_double),
+        ("cfl", C.c_double), ("c_vol", C.c_double),
+        ("dt_growth", C.c_double), ("dt_max", C.c_double), ("dt_init", C.c_double),
+        ("t_stop", C.c_double), ("dt_first", C.c_double), ("t0", C.c_double),
+        ("reflect_mask", C.c_uint32),
+        ("init_kind", C.c_int32),
+        ("rho0", C.c_double), ("e0", C.c_double), ("sedov_energy", C.c_double),
+        ("user", C.POINTER(C.c_double) * 8),
+        ("rank", C.c_int32), ("nranks", C.c_int32), ("device", C.c_int32),
+        ("comm_id", C.c_void_p),
+        ("flags", C.c_uint64),
+    ]
+
+
+class HydroInfoC(C.Structure):
+    _fields_ = [("t", C.c_double), ("dt", C.c_double), ("cycle", C.c_int64),
+                ("dt_min_zone", C.c_double), ("status", C.c_int32), ("bad_zone", C.c_int64)]
+
+
+_lib = None
+
+
+def load_library(path: str = LIB_PATH) -> C.CDLL:
+    """Load the CUDA library; raises (loudly) if it has not been built."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise RuntimeError(f"{path} missing: run __graft_entry__.build() (no CPU fallback exists)")
+    L = C.CDLL(path)
+    L.hydro_config_default.argtypes = [C.POINTER(HydroConfigC)]
+    L.hydro_config_default.restype = None
+    L.hydro_create.argtypes = [C.POINTER(HydroConfigC), C.POINTER(C.c_void_p)]
+    L.hydro_step.argtypes = [C.c_void_p, C.c_int32, C.c_void_p, C.POINTER(HydroInfoC)]
+    L.hydro_get_fields.argtypes = [C.c_void_p, C.c_uint32, C.POINTER(C.POINTER(C.c_double))]
+    L.hydro_get_box.argtypes = [C.c_void_p, C.POINTER(C.c_int64), C.POINTER(C.c_int64),
+                                C.c_uint32, C.POINTER(C.POINTER(C.c_double))]
+    L.hydro_set_state.argtypes = [C.c_void_p, C.POINTER(C.POINTER(C.c_double)),
+                                  C.POINTER(C.c_double), C.c_double, C.c_double]
+    L.hydro_get_info.argtypes = [C.c_void_p, C.POINTER(HydroInfoC)]
+    L.hydro_destroy.argtypes = [C.c_void_p]
+    L.hydro_layout_export.argtypes = [C.POINTER(HydroConfigC), C.POINTER(C.c_int64),
+                                      C.POINTER(C.c_size_t)]
+    L.hydro_decompose_hierarchical.argtypes = [C.POINTER(C.c_int64), C.c_int32, C.c_int32,
+                                               C.POINTER(C.c_int32),
+                                               C.POINTER(C.POINTER(C.c_int64)),
+                                               C.POINTER(C.c_int32)]
+    L.hydro_weighted_slabs.argtypes = [C.c_int64, C.c_int32, C.POINTER(C.c_double),
+                                       C.POINTER(C.c_int64)]
+    L.hydro_comm_unique_id.argtypes = [C.c_void_p]
+    L.hydro_strerror.restype = C.c_char_p
+    L.hydro_last_error.argtypes = [C.c_void_p]
+    L.hydro_last_error.restype = C.c_char_p
+    if L.hydro_abi_version() != ABI_VERSION:
+        raise RuntimeError("libhydro_b200 ABI version mismatch")
+    _lib = L
+    return L
+
+
+@dataclass
+class HydroConfig:
+    """Mirror of hydro_config (include/hydro.h); defaults = hydro_config_default()."""
+    n: Sequence[int] = (32, 32, 32)
+    origin: Sequence[float] = (0.0, 0.0, 0.0)
+    extent: Sequence[float] = (1.2, 1.2, 1.2)
+    ndom: Sequence[int] = (1, 1, 1)
+    cuts: Optional[Sequence[Sequence[int]]] = None
+    dom_to_rank: Optional[Sequence[int]] = None
+    rank_weight: Optional[Sequence[float]] = None
+    gamma: float = 1.4
+    q_lin: float = 0.5
+    q_quad: float = 2.0
+    cfl: float = 0.3
+    c_vol: float = 0.1
+    dt_growth: float = 1.1
+    dt_max: float = math.inf
+    dt_init: float = math.inf
+    t_stop: float = 0.0
+    dt_first: float = 0.0
+    t0: float = 0.0
+    reflect_mask: int = 0x3F
+    init: str = "sedov"          # "sedov" | "user" | "user_mass"
+    rho0: float = 1.0
+    e0: float = 0.0
+    sedov_energy: float = 0.851072 / 8.0
+    user: Optional[Dict[str, np.ndarray]] = None
+    rank: int = 0
+    nranks: int = 1
+    device: int = 0
+    split: bool = False           # HYDRO_FLAG_SPLIT: 3-kernel pipeline instead of fused
+    graph: bool = True            # CUDA graphs (HYDRO_FLAG_NO_GRAPH when False)
+
+
+class HydroError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"hydro error {code} ({STATUS.get(code, '?')}): {msg}")
+        self.code = code
+
+
+def _cfg_struct(cfg: HydroConfig, keep: list, comm_id: Optional[bytes] = None) -> HydroConfigC:
+    L = load_library()
+    c = HydroConfigC()
+    L.hydro_config_default(C.byref(c))
+    for a in range(3):
+        c.n[a] = int(cfg.n[a])
+        c.origin[a] = float(cfg.origin[a])
+        c.extent[a] = float(cfg.extent[a])
+        c.ndom[a] = int(cfg.ndom[a])
+        if cfg.cuts is not None and cfg.cuts[a] is not None:
+            arr = np.ascontiguousarray(cfg.cuts[a], dtype=np.int64)
+            keep.append(arr)
+            c.cuts[a] = arr.ctypes.data_as(C.POINTER(C.c_int64))
+    if cfg.dom_to_rank is not None:
+        arr = np.ascontiguousarray(cfg.dom_to_rank, dtype=np.int32)
+        keep.append(arr)
+        c.dom_to_rank = arr.ctypes.data_as(C.POINTER(C.c_int32))
+    if cfg.rank_weight is not None:
+        arr = np.ascontiguousarray(cfg.rank_weight, dtype=np.float64)
+        keep.append(arr)
+        c.rank_weight = arr.ctypes.data_as(C.POINTER(C.c_double))
+    for k in ("gamma", "q_lin", "q_quad", "cfl", "c_vol", "dt_growth", "dt_max", "dt_init",
+              "t_stop", "dt_first", "t0", "rho0", "e0", "sedov_energy"):
+        setattr(c, k, float(getattr(cfg, k)))
+    c.reflect_mask = int(cfg.reflect_mask)
+    c.init_kind = {"sedov": 0, "user": 1, "user_mass": 2}[cfg.init]
+    if cfg.init != "sedov":
+        names = ("x", "y", "z", "u", "v", "w", "rho" if cfg.init == "user" else "mass", "e")
+        for f, nm in enumerate(names):
+            arr = np.ascontiguousarray(cfg.user[nm], dtype=np.float64).ravel()
+            keep.append(arr)
+            c.user[f] = arr.ctypes.data_as(C.POINTER(C.c_double))
+    c.rank, c.nranks, c.device = int(cfg.rank), int(cfg.nranks), int(cfg.device)
+    if comm_id is not None:
+        buf = C.create_string_buffer(comm_id, 128)
+        keep.append(buf)
+        c.comm_id = C.cast(buf, C.c_void_p)
+    c.flags = (0 if cfg.graph else FLAG_NO_GRAPH) | (FLAG_SPLIT if cfg.split else 0)
+    return c
+
+
+def layout_export(cfg: HydroConfig) -> np.ndarray:
+    """hydro_layout_export: the integer layout (host-only; no GPU needed)."""
+    L = load_library()
+    keep: list = []
+    c = _cfg_struct(cfg, keep)
+    n = C.c_size_t(0)
+    L.hydro_layout_export(C.byref(c), None, C.byref(n))
+    buf = np.zeros(n.value, dtype=np.int64)
+    rc = L.hydro_layout_export(C.byref(c), buf.ctypes.data_as(C.POINTER(C.c_int64)), C.byref(n))
+    if rc != 0:
+        raise HydroError(rc, L.hydro_last_error(None).decode())
+    return buf
+
+
+def decompose_hierarchical(n: Sequence[int], ngpu: int, dpg: int):
+    """hydro_decompose_hierarchical -> (ndom, cuts, dom_to_rank)."""
+    L = load_library()
+    nn = (C.c_int64 * 3)(*[int(v) for v in n])
+    nd = (C.c_int32 * 3)()
+    cuts = [np.zeros(int(v) + 1, dtype=np.int64) for v in n]
+    cptr = (C.POINTER(C.c_int64) * 3)(*[a.ctypes.data_as(C.POINTER(C.c_int64)) for a in cuts])
+    d2r = np.zeros(ngpu * dpg, dtype=np.int32)
+    rc = L.hydro_decompose_hierarchical(nn, int(ngpu), int(dpg), nd, cptr,
+                                        d2r.ctypes.data_as(C.POINTER(C.c_int32)))
+    if rc != 0:
+        raise HydroError(rc, "decompose_hierarchical")
+    ndom = tuple(int(v) for v in nd)
+    return ndom, [cuts[a][: ndom[a] + 1].tolist() for a in range(3)], d2r.tolist()
+
+
+def weighted_slabs(nplanes: int, weights: Sequence[float]):
+    L = load_library()
+    w = np.ascontiguousarray(weights, dtype=np.float64)
+    out = np.zeros(len(w), dtype=np.int64)
+    rc = L.hydro_weighted_slabs(int(nplanes), len(w), w.ctypes.data_as(C.POINTER(C.c_double)),
+                                out.ctypes.data_as(C.POINTER(C.c_int64)))
+    if rc != 0:
+        raise HydroError(rc, "weighted_slabs")
+    return out.tolist()
+
+
+def _info(i: HydroInfoC) -> dict:
+    return {"t": i.t, "dt": i.dt, "cycle": i.cycle, "dt_min_zone": i.dt_min_zone,
+            "status": i.status, "bad_zone": i.bad_zone}
+
+
+class Hydro:
+    """One hydro run on this process's GPU (collective over ranks when nranks > 1)."""
+
+    def __init__(self, cfg: HydroConfig, group=None):
+        self.cfg = cfg
+        self._L = load_library()
+        self._group = group
+        comm_id = None
+        if cfg.nranks > 1:
+            comm_id = self._bootstrap_comm_id()
+        keep: list = []
+        c = _cfg_struct(cfg, keep, comm_id)
+        h = C.c_void_p()
+        rc = self._L.hydro_create(C.byref(c), C.byref(h))
+        if rc != 0:
+            raise HydroError(rc, self._L.hydro_last_error(None).decode())
+        self._h = h
+
+    def _bootstrap_comm_id(self) -> bytes:
+        import torch
+        import torch.distributed as dist
+        buf = bytearray(128)
+        if self.cfg.rank == 0:
+            raw = C.create_string_buffer(128)
+            rc = self._L.hydro_comm_unique_id(raw)
+            if rc != 0:
+                raise HydroError(rc, "hydro_comm_unique_id")
+            buf = bytearray(raw.raw)
+        t = torch.tensor(list(buf), dtype=torch.uint8)
+        if dist.get_backend(self._group) == "nccl":
+            t = t.cuda()
+        dist.broadcast(t, 0, group=self._group)
+        return bytes(t.cpu().tolist())
+
+    def step(self, ncycles: int, stream: Optional[int] = None) -> dict:
+        info = HydroInfoC()
+        rc = self._L.hydro_step(self._h, int(ncycles), C.c_void_p(stream) if stream else None,
+                                C.byref(info))
+        d = _info(info)
+        d["rc"] = rc
+        if rc in (-3, -4, -1):
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+        return d
+
+    def info(self) -> dict:
+        info = HydroInfoC()
+        self._L.hydro_get_info(self._h, C.byref(info))
+        return _info(info)
+
+    def _arrays(self, names, node_shape, zone_shape, alloc=np.zeros):
+        out = {}
+        ptrs = (C.POINTER(C.c_double) * 13)()
+        mask = 0
+        for nm in names:
+            f = ALL_FIELDS.index(nm)
+            arr = alloc(node_shape if f < 6 else zone_shape, dtype=np.float64)
+            out[nm] = arr
+            ptrs[f] = arr.ctypes.data_as(C.POINTER(C.c_double))
+            mask |= 1 << f
+        return out, ptrs, mask
+
+    def fields(self, names: Sequence[str] = ALL_FIELDS) -> Dict[str, np.ndarray]:
+        nx, ny, nz = (int(v) for v in self.cfg.n)
+        out, ptrs, mask = self._arrays(names, (nz + 1, ny + 1, nx + 1), (nz, ny, nx))
+        rc = self._L.hydro_get_fields(self._h, mask, ptrs)
+        if rc != 0:
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+        if self.cfg.nranks > 1:
+            out = self._combine(out)
+        return out
+
+    def box(self, lo: Sequence[int], hi: Sequence[int], names: Sequence[str] = ALL_FIELDS):
+        """Fields of the global zone box [lo, hi) (nodes [lo, hi])."""
+        ext = [int(hi[a]) - int(lo[a]) for a in range(3)]
+        out, ptrs, mask = self._arrays(names, (ext[2] + 1, ext[1] + 1, ext[0] + 1),
+                                       (ext[2], ext[1], ext[0]))
+        clo = (C.c_int64 * 3)(*[int(v) for v in lo])
+        chi = (C.c_int64 * 3)(*[int(v) for v in hi])
+        rc = self._L.hydro_get_box(self._h, clo, chi, mask, ptrs)
+        if rc != 0:
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+        if self.cfg.nranks > 1:
+            out = self._combine(out)
+        return out
+
+    def _combine(self, out):
+        import torch
+        import torch.distributed as dist
+        res = {}
+        for k, v in out.items():
+            t = torch.from_numpy(v)
+            if dist.get_backend(self._group) == "nccl":
+                t = t.cuda()
+            dist.all_reduce(t, group=self._group)  # each entry is written by exactly one rank
+            res[k] = t.cpu().numpy()
+        return res
+
+    def set_state(self, nodes: Dict[str, np.ndarray], e: np.ndarray, t: float, dt: float):
+        arrs = [np.ascontiguousarray(nodes[k], dtype=np.float64) for k in NODE_FIELDS]
+        ea = np.ascontiguousarray(e, dtype=np.float64)
+        ptrs = (C.POINTER(C.c_double) * 6)(*[a.ctypes.data_as(C.POINTER(C.c_double)) for a in arrs])
+        rc = self._L.hydro_set_state(self._h, ptrs, ea.ctypes.data_as(C.POINTER(C.c_double)),
+                                     float(t), float(dt))
+        if rc != 0:
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._L.hydro_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

@@ -1,0 +1,164 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, element by element.
+
+Tolerance (BASELINE.json north_star): relative max-norm per field <= 1e-12 after one cycle,
+<= 1e-10 after 100 cycles (reading R15 defines the norm).  Both sides get the same
+seeded inputs (paper_conf_icppw_pearce18_b200.inputs) or generate the same analytic Sedov state.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle import OracleConfig
+from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig
+from paper_conf_icppw_pearce18_b200.inputs import jittered_state
+from tests.helpers import rel_err, total_energy, user_state
+
+pytestmark = pytest.mark.gpu
+
+FIELDS = ("x", "y", "z", "u", "v", "w", "rho", "e", "p", "q", "c", "vol", "mass")
+PATHS = [False, True]  # split=False: fused default path; split=True: 3-kernel pipeline
+
+
+def run_gpu(ncycles, **kw):
+    with Hydro(HydroConfig(**kw)) as h:
+        info = h.step(ncycles)
+        f = h.fields()
+    return f, info
+
+
+def compare(fg, fo, tol, fields=FIELDS):
+    errs = {k: rel_err(fg[k], fo[k]) for k in fields}
+    bad = {k: v for k, v in errs.items() if not v <= tol}
+    assert not bad, f"fields over {tol}: {bad}"
+    return errs
+
+
+def ocfg(gk):
+    keys = ("n", "origin", "extent", "gamma", "q_lin", "q_quad", "cfl", "c_vol", "dt_growth",
+            "dt_max", "dt_init", "t_stop", "dt_first", "t0", "reflect_mask", "init", "rho0", "e0",
+            "sedov_energy", "user", "ndom", "cuts")
+    return OracleConfig(**{k: v for k, v in gk.items() if k in keys})
+
+
+@pytest.mark.parametrize("split", PATHS)
+def test_sedov32_one_and_hundred_cycles(split):
+    kw = dict(n=(32, 32, 32))
+    for nc, tol in ((1, 1e-12), (100, 1e-10)):
+        fo, io = oracle.run(ocfg(kw), nc)
+        fg, ig = run_gpu(nc, split=split, **kw)
+        assert ig["status"] == 0 and ig["cycle"] == nc
+        compare(fg, fo, tol)
+        assert ig["t"] == pytest.approx(io["t"], rel=tol)
+        assert ig["dt"] == pytest.approx(io["dt"], rel=tol)
+
+
+@pytest.mark.parametrize("split", PATHS)
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_jittered16(seed, split):
+    n = (16, 16, 16)
+    kw = dict(n=n, init="user", user=jittered_state(n, seed))
+    for nc, tol in ((1, 1e-12), (100, 1e-10)):
+        fo, io = oracle.run(ocfg(kw), nc)
+        fg, ig = run_gpu(nc, split=split, **kw)
+        assert ig["status"] == 0
+        compare(fg, fo, tol)
+        assert ig["dt"] == pytest.approx(io["dt"], rel=tol)
+
+
+@pytest.mark.parametrize("split", PATHS)
+def test_ragged_mesh_several_tiles(split):
+    n = (77, 37, 21)  # not a multiple of any tile size; x spans several warps
+    kw = dict(n=n, init="user", user=jittered_state(n, 4))
+    fo, _ = oracle.run(ocfg(kw), 10)
+    fg, ig = run_gpu(10, split=split, **kw)
+    assert ig["status"] == 0
+    compare(fg, fo, 1e-11)
+
+
+@pytest.mark.parametrize("split", PATHS)
+def test_multi_domain_on_one_gpu(split):
+    n = (24, 20, 18)
+    cuts = [[0, 5, 13, 24], [0, 1, 20], [0, 9, 10, 18]]
+    kw = dict(n=n, ndom=(3, 2, 3), cuts=cuts, init="user", user=jittered_state(n, 7))
+    fo, _ = oracle.run(ocfg(kw), 25)
+    fg, ig = run_gpu(25, split=split, **kw)
+    assert ig["status"] == 0
+    compare(fg, fo, 1e-10)
+    single = dict(kw)
+    single.update(ndom=(1, 1, 1), cuts=None)
+    fs, _ = run_gpu(25, split=split, **single)
+    for k in FIELDS:  # same kernels on the same inputs: bitwise
+        assert np.array_equal(fs[k], fg[k]), k
+
+
+@pytest.mark.parametrize("split", PATHS)
+def test_energy_conserved_and_mass_constant(split):
+    kw = dict(n=(24, 24, 24))
+    with Hydro(HydroConfig(split=split, **kw)) as h:
+        f0 = h.fields()
+        h.step(100)
+        f = h.fields()
+    E0 = sum(total_energy(f0))
+    assert abs(sum(total_energy(f)) - E0) / E0 <= 1e-12
+    assert np.array_equal(f["mass"], f0["mass"])
+
+
+@pytest.mark.parametrize("split", PATHS)
+def test_uniform_rest_bitwise(split):
+    n = (8, 8, 8)
+    s = user_state(n, extent=(1.0, 1.0, 1.0))
+    with Hydro(HydroConfig(n=n, extent=(1.0, 1.0, 1.0), init="user", user=s, split=split)) as h:
+        f0 = h.fields()
+        h.step(50)
+        f = h.fields()
+    for k in ("x", "y", "z", "u", "v", "w", "e"):
+        assert np.array_equal(f[k], f0[k]), k
+
+
+def test_t_stop_and_no_op_cycles():
+    kw = dict(n=(16, 16, 16), t_stop=0.01)
+    fo, io = oracle.run(ocfg(kw), 1000)
+    fg, ig = run_gpu(1000, **kw)
+    assert ig["t"] == pytest.approx(0.01, rel=1e-14)
+    assert ig["cycle"] == io["cycle"]
+    compare(fg, fo, 1e-10)
+
+
+def test_tangled_mesh_reported():
+    n = (6, 6, 6)
+    s = user_state(n, e=1.0)
+    s["u"][3, 3, 3] = 1e4
+    with Hydro(HydroConfig(n=n, init="user", user=s, dt_first=1e-3)) as h:
+        r = h.step(5)
+        assert r["rc"] == -5 and r["cycle"] == 1
+        io = oracle.Oracle(ocfg(dict(n=n, init="user", user=s, dt_first=1e-3))).step(5)
+        assert r["bad_zone"] == io["bad_zone"]
+        assert h.step(1)["rc"] == -8
+
+
+def test_restart_set_state_bitwise():
+    kw = dict(n=(16, 12, 10), init="user", user=jittered_state((16, 12, 10), 9))
+    with Hydro(HydroConfig(**kw)) as a:
+        a.step(10)
+        mid = a.fields()
+        ia = a.info()
+        a.step(10)
+        fa = a.fields()
+    with Hydro(HydroConfig(**kw)) as b:
+        b.set_state(mid, mid["e"], ia["t"], ia["dt"])
+        b.step(10)
+        fb = b.fields()
+    for k in FIELDS:
+        assert np.array_equal(fa[k], fb[k]), k
+
+
+def test_full_size_128_against_oracle():
+    """BASELINE.json config 1 (Sedov 128^3, single domain) in the launch configuration bench.py
+    times (fused kernel, CUDA graphs), element by element against the oracle."""
+    kw = dict(n=(128, 128, 128))
+    fo, io = oracle.run(ocfg(kw), 5)
+    fg, ig = run_gpu(5, **kw)
+    compare(fg, fo, 1e-12)
+    assert ig["dt"] == pytest.approx(io["dt"], rel=1e-12)
