@@ -1,0 +1,347 @@
+"""Benchmark: zone-cycles/s of the fp64 Lagrangian hydro cycle (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config sedov128] [--impl ours|reference]
+
+A "step" is one full cycle of the hot path (S1-S9: fused cycle kernel, halo, dt reduction) over
+the whole mesh.  N=1 default workload: BASELINE.json configs[1], "Sedov blast 3D 128^3 zones,
+single domain on 1xB200".  For N > 1 (torchrun, one process per GPU) the per-GPU work is fixed
+(weak scaling): 128^3 zones per GPU, the global mesh split by the hierarchical rule (PAPER.md
+L559-572).  Other BASELINE configs are selectable with --config.
+
+value: zone-cycles/s over all ranks, device-timed with CUDA events on the launching stream,
+max over ranks.  e2e: the same metric through the public API with host buffers (set_state
+H2D + 100 cycles + get_fields D2H per e2e step).  roofline: the fused cycle kernel's
+algorithmic bytes / its mean duration (hydro_time_kernels, CUDA events) against the measured
+HBM copy bandwidth.  cpu_baseline / --impl reference: the oracle (test infrastructure) on the
+host cores, on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    # name: (description, per-GPU or global mesh rule)
+    "sedov32": "Sedov blast 3D 32^3 zones, single domain, 100 cycles fp64",
+    "sedov128": "Sedov blast 3D 128^3 zones, single domain on 1xB200",
+    "sedov512": "Sedov blast 3D 512^3 zones strong-scaled, 8 domains over N B200",
+    "weak384": "weak scaling 384^3 zones per GPU, 4 y-slab domains per GPU",
+    "uneven448": "unevenly sized domains 3D 448^3, cuts {0,64,160,288,448}, LPT onto N GPUs",
+}
+METRIC = "zone-cycles/sec fp64"
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def hier(n, ngpu, dpg):
+    from paper_conf_icppw_pearce18_b200 import decompose_hierarchical
+    return decompose_hierarchical(n, ngpu, dpg)
+
+
+def workload(name: str, ngpu: int):
+    """Return (HydroConfig kwargs, scaling, description)."""
+    h = 1.2 / 128
+    if name in ("sedov128", "sedov32"):
+        base = 128 if name == "sedov128" else 32
+        if ngpu == 1:
+            return dict(n=(base,) * 3), "weak", CONFIGS[name]
+        ndom, cuts, d2r = hier((base, base, base), ngpu, 1)
+        n = tuple(base * ndom[a] for a in range(3))
+        ndom, cuts, d2r = hier(n, ngpu, 1)
+        hb = 1.2 / base
+        return (dict(n=n, extent=tuple(hb * v for v in n), ndom=ndom, cuts=cuts, dom_to_rank=d2r),
+                "weak", f"Sedov blast 3D {base}^3 zones per GPU (weak), global {n}, {ngpu} domains")
+    if name == "sedov512":
+        n = (512, 512, 512)
+        ndom, cuts, d2r = hier(n, ngpu, 8 // ngpu) if ngpu in (1, 2, 4, 8) else hier(n, ngpu, 1)
+        return dict(n=n, ndom=ndom, cuts=cuts, dom_to_rank=d2r), "strong", CONFIGS[name]
+    if name == "weak384":
+        gshape = {1: (1, 1, 1), 2: (2, 1, 1), 4: (2, 2, 1), 8: (2, 2, 2)}.get(ngpu)
+        n = tuple(384 * g for g in gshape)
+        ndom, cuts, d2r = hier(n, ngpu, 4)
+        hb = 1.2 / 384
+        return (dict(n=n, extent=tuple(hb * v for v in n), ndom=ndom, cuts=cuts, dom_to_rank=d2r),
+                "weak", CONFIGS[name])
+    if name == "uneven448":
+        c = [0, 64, 160, 288, 448]
+        return dict(n=(448,) * 3, ndom=(4, 4, 4), cuts=[c, c, c]), "strong", CONFIGS[name]
+    raise SystemExit(f"unknown config {name}")
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons with NVML during the timed region."""
+
+    def __init__(self, device: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        try:
+            import pynvml as N
+            N.nvmlInit()
+            self.N = N
+            self.hdl = N.nvmlDeviceGetHandleByIndex(device)
+            self.max_mhz = N.nvmlDeviceGetMaxClockInfo(self.hdl, N.NVML_CLOCK_SM)
+        except Exception:
+            self.N = None
+
+    def _run(self):
+        N = self.N
+        names = {
+            "gpu_idle": 0x1, "applications_clocks_setting": 0x2, "sw_power_cap": 0x4,
+            "hw_slowdown": 0x8, "sync_boost": 0x10, "sw_thermal_slowdown": 0x20,
+            "hw_thermal_slowdown": 0x40, "hw_power_brake_slowdown": 0x80,
+        }
+        while not self._stop.is_set():
+            try:
+                self.samples.append(N.nvmlDeviceGetClockInfo(self.hdl, N.NVML_CLOCK_SM))
+                r = N.nvmlDeviceGetCurrentClocksEventReasons(self.hdl)
+                for k, bit in names.items():
+                    if r & bit and k != "gpu_idle":
+                        self.reasons.add(k)
+            except Exception:
+                pass
+            time.sleep(0.02)
+
+    def __enter__(self):
+        if self.N:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.N:
+            self.t.join()
+
+    def summary(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(self.samples)}
+
+
+def measured_peak_hbm():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def fp64_peak():
+    """Measured DFMA lane-op rate (profiles/r01_fp64_peak.txt, tools/fp64_peak.cu)."""
+    return 1.708e13
+
+
+def oracle_baseline(kw, budget_s=12.0):
+    """Time the oracle (as it stands) on a bounded sample of the workload on this host."""
+    import oracle
+    from oracle import OracleConfig
+    n = kw.get("n")
+    sample_n = n
+    # one cycle of the whole mesh if it fits the budget (~3 M zone-cycles/s), else a sub-box
+    zones = n[0] * n[1] * n[2]
+    if zones > 2_200_000:
+        s = int(round((2_097_152) ** (1.0 / 3.0)))
+        sample_n = (s, s, s)
+        zones = s ** 3
+    cfg = OracleConfig(n=sample_n, extent=tuple(1.2 / 128 * v for v in sample_n)
+                       if sample_n != (128, 128, 128) else (1.2, 1.2, 1.2))
+    o = oracle.Oracle(cfg)
+    o.step(1)  # warm
+    t0 = time.perf_counter()
+    cycles = 0
+    while True:
+        o.step(1)
+        cycles += 1
+        el = time.perf_counter() - t0
+        if el > budget_s or cycles >= 100:
+            break
+    o.close()
+    return {"value": zones * cycles / el, "unit": METRIC, "cores": 1, "kind": "oracle",
+            "sample": f"Sedov {sample_n[0]}x{sample_n[1]}x{sample_n[2]}, {cycles} cycles "
+                      f"single-threaded after 1 warm-up cycle ({el:.1f} s)"}
+
+
+def run_reference(args):
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return
+    kw, scaling, desc = workload(args.config, max(ws, args.gpus))
+    import oracle
+    from oracle import OracleConfig
+    n = kw["n"]
+    zones = n[0] * n[1] * n[2]
+    # bounded sample: the whole mesh if a step is cheap, else a 64^3 Sedov sub-problem per step
+    per_cycle_s = zones / 3.0e6
+    sample_n = n if per_cycle_s * (args.steps + args.warmup) < 150 else (64, 64, 64)
+    sz = sample_n[0] * sample_n[1] * sample_n[2]
+    o = oracle.Oracle(OracleConfig(n=sample_n, extent=kw.get("extent", (1.2,) * 3)
+                                   if sample_n == n else (1.2 / 128 * 64,) * 3))
+    o.step(args.warmup)
+    t0 = time.perf_counter()
+    o.step(args.steps)
+    el = time.perf_counter() - t0
+    o.close()
+    v = sz * args.steps / el
+    line = {"metric": METRIC, "value": v, "unit": "zone-cycles/s", "impl": "reference",
+            "n_gpus": 0, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * el / args.steps, "higher_is_better": True, "scaling": scaling,
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": desc, "sample": list(sample_n)},
+            "cpu_baseline": {"value": v, "unit": "zone-cycles/s", "cores": 1, "kind": "oracle",
+                             "sample": f"Sedov {sample_n}, {args.steps} cycles per run"},
+            "e2e": {"value": v, "unit": "zone-cycles/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--config", default="sedov128", choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--split", action="store_true", help="3-kernel split pipeline")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-cycles", type=int, default=100)
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    args.warmup = max(args.warmup, 3)
+
+    import numpy as np
+    import torch
+
+    ws, rank, local = dist_env()
+    ngpu = max(ws, 1)
+    torch.cuda.set_device(local)
+    dist = None
+    if ws > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl")
+    from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig
+
+    kw, scaling, desc = workload(args.config, ngpu)
+    cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, split=args.split, **kw)
+    hyd = Hydro(cfg)
+    n = kw["n"]
+    zones = n[0] * n[1] * n[2]
+    stream = torch.cuda.current_stream()
+    sp = stream.cuda_stream
+
+    def barrier():
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    hyd.step(args.warmup, stream=sp)
+    barrier()
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        start.record(stream)
+        info = hyd.step(args.steps, stream=sp)
+        end.record(stream)
+        torch.cuda.synchronize()
+    ms = start.elapsed_time(end)
+    if dist:
+        t = torch.tensor([ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    barrier()
+    value = zones * args.steps / (ms * 1e-3)
+    if info["status"] != 0:
+        raise SystemExit(f"run failed: {info}")
+
+    # per-kernel live timing of the dominant kernel (no graph; CUDA events on the same stream)
+    kt = hyd.time_kernels(min(args.steps, 50))
+    launches = hyd.kernels_per_cycle() * args.steps
+    if dist:
+        t = torch.tensor([launches], device="cuda", dtype=torch.float64)
+        dist.all_reduce(t)
+        launches = int(t.item())
+
+    # algorithmic bytes of one fused-kernel launch on this rank: read + write of
+    # x,u (6 doubles) on the domain's nodes, read m,e and write e on its zones
+    local_doms = [d for d in range(int(np.prod(cfg.ndom)))
+                  if (kw.get("dom_to_rank") or [0] * 512)[d] == rank] if ngpu > 1 else [0]
+    nd_local = len(local_doms) if ngpu > 1 else int(np.prod(cfg.ndom))
+    z_rank = zones // ngpu if scaling == "weak" or ngpu > 1 else zones
+    per_dom_z = z_rank / max(nd_local, 1)
+    side = per_dom_z ** (1.0 / 3.0)
+    per_dom_nodes = (side + 1) ** 3
+    alg_bytes = 96.0 * per_dom_nodes + 24.0 * per_dom_z
+    peak, peak_kind = measured_peak_hbm()
+    achieved = alg_bytes / (kt["cycle_kernel_ms"] * 1e-3) / 1e9
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+            "frac": achieved / peak, "traffic": None, "peak_source": peak_kind,
+            "kernel": "k_cycle_fused" if not args.split else "split zone+node+energy",
+            "kernel_ms": kt["cycle_kernel_ms"], "kernel_share_of_cycle":
+            kt["cycle_kernel_ms"] * nd_local / kt["cycle_ms"] if kt["cycle_ms"] else None,
+            "alg_bytes_per_launch": alg_bytes}
+
+    # end to end through the public API with host buffers: H2D state, e2e_cycles cycles, D2H
+    e2e = None
+    if ngpu == 1:
+        names = ("x", "y", "z", "u", "v", "w", "e")
+        cur = hyd.fields(names)
+        pinned = {k: torch.from_numpy(v).pin_memory().numpy() for k, v in cur.items()}
+        out = {k: torch.empty(v.shape, dtype=torch.float64).pin_memory().numpy()
+               for k, v in cur.items()}
+        inf0 = hyd.info()
+        reps = 3
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            hyd.set_state(pinned, pinned["e"], inf0["t"], inf0["dt"])
+            hyd.step(args.e2e_cycles)
+            got = hyd.fields(names)
+            for k in names:
+                out[k][...] = got[k]
+        el = time.perf_counter() - t0
+        h2d = sum(v.nbytes for v in pinned.values())
+        d2h = sum(v.nbytes for v in out.values())
+        e2e = {"value": zones * args.e2e_cycles * reps / el, "unit": "zone-cycles/s",
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "cycles_per_step": args.e2e_cycles,
+               "note": "per e2e step: hydro_set_state (H2D) + hydro_step(cycles) + hydro_get_fields (D2H)"}
+    cpu = None
+    if rank == 0 and ngpu == 1 and not args.no_cpu_baseline:
+        cpu = oracle_baseline(kw)
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "zone-cycles/s", "n_gpus": ngpu,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": desc, "mesh": list(n), "domains": list(cfg.ndom),
+                       "zones": zones, "path": "split" if args.split else "fused",
+                       "l2": "state > 126 MB L2 (inputs larger than L2; no flush)"
+                       if zones * 120 > 126e6 else "state fits L2",
+                       "parallelism": f"dp{ngpu} (spatial domains)"},
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk.summary(),
+            "gpu_launches": launches, "kernel_ms": kt,
+        }
+        print(json.dumps(line), flush=True)
+    hyd.close()
+    if dist:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -151,6 +151,16 @@ int hydro_get_info(hydro_ctx *h, hydro_info *info);
 /* Destroy; NULL-safe; collective. */
 int hydro_destroy(hydro_ctx *h);
 
+/* Measurement helper (bench.py): run ncycles cycles WITHOUT CUDA graphs on the context stream,
+   bracketing each kernel class with CUDA events, and report mean device milliseconds:
+   out_ms[0] per cycle-kernel launch (fused kernel, or zone+node+energy of one domain when split),
+   out_ms[1] halo exchange per cycle, out_ms[2] dt finalize per cycle, out_ms[3] whole cycle.
+   Advances the state like hydro_step.  Collective. */
+int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[4]);
+
+/* Number of kernels of this library launched per cycle on this rank (bench.py gpu_launches). */
+int hydro_kernels_per_cycle(const hydro_ctx *h);
+
 /* --- host-only helpers (no CUDA device needed) --------------------------------------------- */
 
 /* Build the integer layout for cfg without touching the GPU and serialise it as int64 words

@@ -186,6 +186,10 @@ int comm_status_agree(Comm *c, int status) {
   return v;
 }
 
+int comm_kernels_per_cycle(const Comm *c) {
+  return (c->sends.empty() ? 0 : 1) + (c->recvs.empty() ? 0 : 1);
+}
+
 void comm_destroy(Comm *c) {
   if (!c) return;
   if (c->nccl) ncclCommDestroy(c->nccl);

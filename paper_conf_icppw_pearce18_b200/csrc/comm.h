@@ -31,6 +31,7 @@ int comm_dt_min(Comm *c, unsigned long long *dev_bits, cudaStream_t s);
 int comm_halo(Comm *c, int par, cudaStream_t s);
 // Agree on a status code across ranks (the most negative wins).
 int comm_status_agree(Comm *c, int status);
+int comm_kernels_per_cycle(const Comm *c);
 void comm_destroy(Comm *c);
 
 }  // namespace hydro

@@ -1,8 +1,11 @@
 // kernels.h -- host-side launchers for the CUDA kernels (all enqueue on `s`, never synchronise).
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include "device.cuh"
+
+#define FUSED_BOX_X 36  // TMA node box width (TX + 3 = 35 rounded up to a 16-byte row)
 
 namespace hydro {
 
@@ -28,8 +31,16 @@ void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, cudaStrea
 void launch_node_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 void launch_energy_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 
+// TMA descriptors of the six node-state arrays (x,y,z,u,v,w) of one domain and parity.
+struct alignas(64) NodeMaps {
+  CUtensorMap m[6];
+};
+
 // Fused single-kernel cycle (default path).
-void launch_cycle_fused(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
+                        cudaStream_t s);
+size_t fused_smem_bytes();
+int fused_box_y();
 
 // End of cycle: S9 dt / time update and error latch.
 void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s);

@@ -1,6 +1,8 @@
 // runtime.cu -- the C ABI of include/hydro.h: context, per-domain device allocation, CUDA-graph
 // capture of a cycle, host<->device field transfer.  One process drives one GPU; all domains
 // assigned to this rank live in its HBM (each rank owns its domains).
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -28,6 +30,7 @@ struct LocalDom {
   void *mem = nullptr;
   size_t bytes = 0;
   DomView view[2];  // parity p reads view[p].x and writes view[p].xn
+  NodeMaps maps[2]; // TMA descriptors of view[p]'s current node arrays
 };
 
 }  // namespace
@@ -72,8 +75,9 @@ size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 
 int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
   const int64_t n0 = D.box.n[0], n1 = D.box.n[1], n2 = D.box.n[2];
-  const int64_t nsx = n0 + 3, nsxy = nsx * (n1 + 3), nnode = nsxy * (n2 + 3);
-  const int64_t zsx = n0 + 2, zsxy = zsx * (n1 + 2), nzone = zsxy * (n2 + 2);
+  // row pitches padded to 4 doubles (32 B): TMA needs 16-byte strides
+  const int64_t nsx = (n0 + 3 + 3) / 4 * 4, nsxy = nsx * (n1 + 3), nnode = nsxy * (n2 + 3);
+  const int64_t zsx = (n0 + 2 + 3) / 4 * 4, zsxy = zsx * (n1 + 2), nzone = zsxy * (n2 + 2);
   const size_t nb = align_up(nnode * sizeof(double), 256), zb = align_up(nzone * sizeof(double), 256);
   // 12 node arrays (2 parities x 6), e x2, m, P, aux x5, optional B x24
   size_t bytes = 12 * nb + 9 * zb + (split ? 24 * zb : 0);
@@ -106,6 +110,32 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
     v.en = par ? e0 : e1;
     v.m = m; v.P = P; v.B = B; v.aux = aux;
     v.dom = D.dom;
+  }
+  // TMA descriptors (3-D tiled, fp64, box FUSED_BOX_X x (TY+3) x 1; out-of-bounds zero fill)
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  if (!encode) {
+    cudaDriverEntryPointQueryResult q;
+    void *fn = nullptr;
+    CK(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
+    if (!fn || q != cudaDriverEntryPointSuccess)
+      return set_err(h, HYDRO_ECUDA, "cuTensorMapEncodeTiled unavailable");
+    encode = (PFN_cuTensorMapEncodeTiled_v12000)fn;
+  }
+  for (int par = 0; par < 2; ++par) {
+    const double *arr[6] = {D.view[par].x, D.view[par].y, D.view[par].z,
+                            D.view[par].u, D.view[par].v, D.view[par].w};
+    for (int f = 0; f < 6; ++f) {
+      cuuint64_t dims[3] = {(cuuint64_t)nsx, (cuuint64_t)(n1 + 3), (cuuint64_t)(n2 + 3)};
+      cuuint64_t strides[2] = {(cuuint64_t)(nsx * sizeof(double)),
+                               (cuuint64_t)(nsxy * sizeof(double))};
+      cuuint32_t box[3] = {FUSED_BOX_X, (cuuint32_t)fused_box_y(), 1};
+      cuuint32_t es[3] = {1, 1, 1};
+      CUresult r = encode(&D.maps[par].m[f], CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3,
+                          const_cast<double *>(arr[f]), dims, strides, box, es,
+                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                          CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      if (r != CUDA_SUCCESS) return set_err(h, HYDRO_ECUDA, "cuTensorMapEncodeTiled failed");
+    }
   }
   return HYDRO_OK;
 }
@@ -191,7 +221,7 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
     for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
     for (LocalDom &D : h->doms) launch_energy_split(D.view[par], h->ph, h->st, s);
   } else {
-    for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], h->ph, h->st, s);
+    for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, s);
     if (h->comm) {
       int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
@@ -332,7 +362,7 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
   h->ph.dt_max = cfg->dt_max;
   h->ph.t_stop = cfg->t_stop;
   h->ph.reflect_mask = cfg->reflect_mask;
-  h->split = true;  // TEMP: fused kernel not yet in tree
+  h->split = (cfg->flags & HYDRO_FLAG_SPLIT) != 0;
   h->use_graph = (cfg->flags & HYDRO_FLAG_NO_GRAPH) == 0;
   h->device = cfg->device;
   *out = nullptr;
@@ -575,6 +605,63 @@ int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, 
   CK(cudaStreamSynchronize(h->stream));
   h->failed = 0;
   return HYDRO_OK;
+}
+
+int hydro_kernels_per_cycle(const hydro_ctx *h) {
+  if (!h) return HYDRO_EINVAL;
+  const int nd = (int)h->doms.size();
+  int k = h->split ? 3 * nd : nd;   // cycle kernels
+  if (h->n_local_pairs > 0) k += 1;  // intra-GPU halo copy
+  k += 1;                            // finalize
+  if (h->comm) k += comm_kernels_per_cycle(h->comm);
+  return k;
+}
+
+int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[4]) {
+  if (!h || ncycles <= 0 || !out_ms) return set_err(h, HYDRO_EINVAL, "bad argument");
+  if (h->failed) return set_err(h, HYDRO_ESTATE, "context failed earlier");
+  CK(cudaSetDevice(h->device));
+  cudaStream_t s = h->stream;
+  cudaEvent_t ev[5];
+  for (int i = 0; i < 5; ++i) CK(cudaEventCreate(&ev[i]));
+  double acc[4] = {0, 0, 0, 0};
+  for (int32_t c = 0; c < ncycles; ++c) {
+    const int par = h->parity;
+    CK(cudaEventRecord(ev[0], s));
+    if (h->split) {
+      for (LocalDom &D : h->doms) launch_zone_split(D.view[par], h->ph, h->st, s);
+      if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
+      for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
+      for (LocalDom &D : h->doms) launch_energy_split(D.view[par], h->ph, h->st, s);
+    } else {
+      for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, s);
+      if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
+    }
+    CK(cudaEventRecord(ev[1], s));
+    launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
+    if (h->comm && comm_halo(h->comm, par, s)) return HYDRO_ENCCL;
+    CK(cudaEventRecord(ev[2], s));
+    launch_finalize(h->st, h->ph, s);
+    CK(cudaEventRecord(ev[3], s));
+    CK(cudaEventSynchronize(ev[3]));
+    float a, b, cc, d;
+    CK(cudaEventElapsedTime(&a, ev[0], ev[1]));
+    CK(cudaEventElapsedTime(&b, ev[1], ev[2]));
+    CK(cudaEventElapsedTime(&cc, ev[2], ev[3]));
+    CK(cudaEventElapsedTime(&d, ev[0], ev[3]));
+    acc[0] += a; acc[1] += b; acc[2] += cc; acc[3] += d;
+    h->parity ^= 1;
+  }
+  for (int i = 0; i < 5; ++i) cudaEventDestroy(ev[i]);
+  const double nd = h->doms.empty() ? 1.0 : (double)h->doms.size();
+  out_ms[0] = acc[0] / ncycles / nd;
+  out_ms[1] = acc[1] / ncycles;
+  out_ms[2] = acc[2] / ncycles;
+  out_ms[3] = acc[3] / ncycles;
+  hydro_info info;
+  const int status = read_info(h, &info, s);
+  if (status < 0 && status != HYDRO_ECUDA) h->failed = status;
+  return status;
 }
 
 int hydro_destroy(hydro_ctx *h) {

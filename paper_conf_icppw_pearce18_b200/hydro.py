@@ -89,6 +89,8 @@ def load_library(path: str = LIB_PATH) -> C.CDLL:
     L.hydro_weighted_slabs.argtypes = [C.c_int64, C.c_int32, C.POINTER(C.c_double),
                                        C.POINTER(C.c_int64)]
     L.hydro_comm_unique_id.argtypes = [C.c_void_p]
+    L.hydro_time_kernels.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_double)]
+    L.hydro_kernels_per_cycle.argtypes = [C.c_void_p]
     L.hydro_strerror.restype = C.c_char_p
     L.hydro_last_error.argtypes = [C.c_void_p]
     L.hydro_last_error.restype = C.c_char_p
@@ -268,6 +270,18 @@ class Hydro:
         if rc in (-3, -4, -1):
             raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
         return d
+
+    def time_kernels(self, ncycles: int) -> dict:
+        """hydro_time_kernels: per-kernel-class mean device ms (no graphs, CUDA events)."""
+        out = (C.c_double * 4)()
+        rc = self._L.hydro_time_kernels(self._h, int(ncycles), out)
+        if rc in (-3, -4, -1, -8):
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+        return {"cycle_kernel_ms": out[0], "halo_ms": out[1], "finalize_ms": out[2],
+                "cycle_ms": out[3]}
+
+    def kernels_per_cycle(self) -> int:
+        return int(self._L.hydro_kernels_per_cycle(self._h))
 
     def info(self) -> dict:
         info = HydroInfoC()
