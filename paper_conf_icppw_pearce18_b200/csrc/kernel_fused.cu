@@ -46,9 +46,10 @@ struct Tile {
   static constexpr int OFF_G = OFF_M + ZS;          // [9][ZS] g_x, g_y, g_z
   static constexpr int OFF_UH = OFF_G + 9 * ZS;     // [2 planes][3][ZS] u_half
   static constexpr int OFF_PS = OFF_UH + 6 * ZS;    // [2][ZS] psi of x-low, y-low faces
-  static constexpr int OFF_BAR = OFF_PS + 2 * ZS;   // 3 mbarriers
+  static constexpr int OFF_RED = OFF_PS + 2 * ZS;   // [32] block dt reduction
+  static constexpr int OFF_BAR = OFF_RED + 32;      // 3 mbarriers
   static constexpr int TOTAL = OFF_BAR + 4;
-  static constexpr size_t BYTES = sizeof(double) * TOTAL + 128;
+  static constexpr size_t BYTES = sizeof(double) * TOTAL;
   static_assert(BXN >= TX + 3, "TMA box too narrow");
   static_assert(BYN <= 256 && BXN <= 256, "TMA box limit");
 };
@@ -94,9 +95,9 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
     k_cycle_fused(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st,
                   int KZ) {
   using T = Tile<TX, TY>;
-  extern __shared__ __align__(128) double sm_raw[];
-  double *sm = reinterpret_cast<double *>((reinterpret_cast<uintptr_t>(sm_raw) + 127) &
-                                          ~uintptr_t(127));
+  // dynamic shared memory only (no static __shared__ in this kernel), so the window starts
+  // 1024-byte aligned and every TMA destination (multiples of 128 B) is aligned
+  extern __shared__ __align__(1024) double sm[];
   double *RAW = sm + T::OFF_RAW, *XP = sm + T::OFF_XP, *PS = sm + T::OFF_P, *MS = sm + T::OFF_M;
   double *GX = sm + T::OFF_G, *GY = GX + 3 * T::ZS, *GZ = GY + 3 * T::ZS;
   double *UH = sm + T::OFF_UH, *PSX = sm + T::OFF_PS, *PSY = PSX + T::ZS;
@@ -159,6 +160,7 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
   };
 
   if (t == 0) {
+    if (smem_u32(sm) & 127u) __trap();  // TMA destinations must be 128-byte aligned
     for (int s = 0; s < 3; ++s) mbar_init(&bar[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     issue(q0);
@@ -393,7 +395,7 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
     bxp = bx0; byp = by0; bzp = bz0;
   }
   // S9 (block part): dt = sqrt(min dt^2), one atomicMin per block.
-  block_min_dt(sqrt(dt2min), &st->dtz_acc);
+  block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);
 }
 
 constexpr int FTX = 32, FTY = 12;

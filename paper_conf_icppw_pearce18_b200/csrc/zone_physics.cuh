@@ -91,9 +91,9 @@ __device__ __forceinline__ ZoneEos zone_eos(double V, double A2max, double DV, d
   return r;
 }
 
-// Warp + block min of a non-negative double, one atomicMin on its bit pattern per block.
-__device__ __forceinline__ void block_min_dt(double v, unsigned long long *acc) {
-  __shared__ double red[32];
+// Warp + block min of a non-negative double, one atomicMin on its bit pattern per block;
+// red: 32 doubles of shared scratch.
+__device__ __forceinline__ void block_min_dt_smem(double v, unsigned long long *acc, double *red) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v = fmin(v, __shfl_xor_sync(0xffffffffu, v, o));
   const int tid = threadIdx.x + blockDim.x * (threadIdx.y + blockDim.y * threadIdx.z);
@@ -107,6 +107,11 @@ __device__ __forceinline__ void block_min_dt(double v, unsigned long long *acc) 
     for (int o = 16; o > 0; o >>= 1) v = fmin(v, __shfl_xor_sync(0xffffffffu, v, o));
     if (lane == 0 && v < INFINITY) atomicMin(acc, (unsigned long long)__double_as_longlong(v));
   }
+}
+
+__device__ __forceinline__ void block_min_dt(double v, unsigned long long *acc) {
+  __shared__ double red[32];
+  block_min_dt_smem(v, acc, red);
 }
 
 }  // namespace hydro
