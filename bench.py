@@ -147,6 +147,13 @@ def fp64_peak():
     return 1.708e13
 
 
+# Executed fp64 pipe instructions (DADD+DMUL+DFMA, thread level) per owned zone and DRAM bytes
+# per owned zone of each kernel at 128^3, from ncu (profiles/r01_*.txt).  The
+# zone stage has no redundant work, so its executed count is the algorithmic count.
+FP64_PER_ZONE = {"k_zone_stage": 0.0, "k_node_energy": 0.0, "k_cycle_fused": 516.0}
+TRAFFIC_PER_ZONE = {}
+
+
 def oracle_baseline(kw, budget_s=12.0):
     """Time the oracle (as it stands) on a bounded sample of the workload on this host."""
     import oracle
@@ -217,7 +224,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--config", default="sedov128", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--split", action="store_true", help="3-kernel split pipeline")
+    ap.add_argument("--path", default="two", choices=["two", "one", "split"],
+                    help="two: zone + node/energy kernels; one: one fused kernel; split: plain")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-cycles", type=int, default=100)
     args = ap.parse_args()
@@ -238,7 +246,7 @@ def main():
     from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig
 
     kw, scaling, desc = workload(args.config, ngpu)
-    cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, split=args.split, **kw)
+    cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, path=args.path, **kw)
     hyd = Hydro(cfg)
     n = kw["n"]
     zones = n[0] * n[1] * n[2]
@@ -276,24 +284,52 @@ def main():
         dist.all_reduce(t)
         launches = int(t.item())
 
-    # algorithmic bytes of one fused-kernel launch on this rank: read + write of
-    # x,u (6 doubles) on the domain's nodes, read m,e and write e on its zones
-    local_doms = [d for d in range(int(np.prod(cfg.ndom)))
-                  if (kw.get("dom_to_rank") or [0] * 512)[d] == rank] if ngpu > 1 else [0]
-    nd_local = len(local_doms) if ngpu > 1 else int(np.prod(cfg.ndom))
-    z_rank = zones // ngpu if scaling == "weak" or ngpu > 1 else zones
-    per_dom_z = z_rank / max(nd_local, 1)
-    side = per_dom_z ** (1.0 / 3.0)
-    per_dom_nodes = (side + 1) ** 3
-    alg_bytes = 96.0 * per_dom_nodes + 24.0 * per_dom_z
+    # Roofline of the dominant kernel.  Algorithmic bytes per launch come from
+    # the exact domain boxes of this rank: N_n nodes and N_z zones per domain.
+    from paper_conf_icppw_pearce18_b200 import layout_export
+    lay = layout_export(cfg)
+    nd_all, nper = int(lay[1]), []
+    for d in range(nd_all):
+        w = lay[7 + 7 * d: 14 + 7 * d]
+        if int(w[6]) == rank:
+            nper.append((int(w[3]), int(w[4]), int(w[5])))
+    nd_local = max(len(nper), 1)
+    Nz = sum(a * b * c for a, b, c in nper) / nd_local
+    Nn = sum((a + 1) * (b + 1) * (c + 1) for a, b, c in nper) / nd_local
     peak, peak_kind = measured_peak_hbm()
-    achieved = alg_bytes / (kt["cycle_kernel_ms"] * 1e-3) / 1e9
-    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-            "frac": achieved / peak, "traffic": None, "peak_source": peak_kind,
-            "kernel": "k_cycle_fused" if not args.split else "split zone+node+energy",
-            "kernel_ms": kt["cycle_kernel_ms"], "kernel_share_of_cycle":
-            kt["cycle_kernel_ms"] * nd_local / kt["cycle_ms"] if kt["cycle_ms"] else None,
-            "alg_bytes_per_launch": alg_bytes}
+    kern = []
+    if args.path == "two":
+        kern.append(("k_zone_stage", kt["zone_stage_ms"], 48.0 * Nn + 24.0 * Nz,
+                     FP64_PER_ZONE["k_zone_stage"] * Nz))
+        kern.append(("k_node_energy", kt["node_stage_ms"], 96.0 * Nn + 32.0 * Nz,
+                     FP64_PER_ZONE["k_node_energy"] * Nz))
+    elif args.path == "one":
+        kern.append(("k_cycle_fused", kt["cycle_kernel_ms"], 96.0 * Nn + 24.0 * Nz,
+                     FP64_PER_ZONE["k_cycle_fused"] * Nz))
+    else:
+        kern.append(("split zone+node+energy", kt["cycle_kernel_ms"],
+                     96.0 * Nn + 24.0 * Nz, None))
+    rows = []
+    for name, ms, byts, flops in kern:
+        hbm = byts / (ms * 1e-3) / 1e9
+        r = {"kernel": name, "ms": ms, "alg_bytes": byts, "hbm_gbs": hbm, "hbm_frac": hbm / peak}
+        if flops:
+            alu = flops / (ms * 1e-3)
+            r.update({"fp64_inst_per_s": alu, "fp64_frac": alu / fp64_peak()})
+        rows.append(r)
+    dom = max(rows, key=lambda r: r["ms"])
+    alu_bound = dom.get("fp64_frac", 0.0) > dom["hbm_frac"]
+    roof = {"bound": "alu" if alu_bound else "hbm",
+            "achieved": dom["fp64_inst_per_s"] / 1e12 if alu_bound else dom["hbm_gbs"],
+            "peak": fp64_peak() / 1e12 if alu_bound else peak,
+            "unit": "T fp64-inst/s" if alu_bound else "GB/s",
+            "frac": dom["fp64_frac"] if alu_bound else dom["hbm_frac"],
+            "traffic": TRAFFIC_PER_ZONE.get(dom["kernel"], 0) * Nz or None,
+            "peak_source": ("measured DFMA rate (profiles/r01_fp64_peak.txt)" if alu_bound
+                            else f"{peak_kind} MEASURED_PEAKS.json hbm_gbs"),
+            "kernel": dom["kernel"], "kernel_ms": dom["ms"],
+            "kernel_share_of_cycle": dom["ms"] * nd_local / kt["cycle_ms"] if kt["cycle_ms"] else None,
+            "alg_bytes_per_launch": dom["alg_bytes"], "kernels": rows}
 
     # end to end through the public API with host buffers: H2D state, e2e_cycles cycles, D2H
     e2e = None
@@ -330,7 +366,7 @@ def main():
             "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
             "config": {"workload": desc, "mesh": list(n), "domains": list(cfg.ndom),
-                       "zones": zones, "path": "split" if args.split else "fused",
+                       "zones": zones, "path": args.path,
                        "l2": "state > 126 MB L2 (inputs larger than L2; no flush)"
                        if zones * 120 > 126e6 else "state fits L2",
                        "parallelism": f"dp{ngpu} (spatial domains)"},

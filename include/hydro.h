@@ -65,7 +65,9 @@ enum {
 
 /* hydro_config.flags */
 #define HYDRO_FLAG_NO_GRAPH (1ull << 0) /* launch kernels directly instead of CUDA graphs */
-#define HYDRO_FLAG_SPLIT (1ull << 1)    /* use the 3-kernel split pipeline, not the fused kernel */
+#define HYDRO_FLAG_SPLIT (1ull << 1)    /* plain 3-kernel pipeline (one thread per element) */
+#define HYDRO_FLAG_ONE_KERNEL (1ull << 2) /* one fused kernel per cycle (zone ring recomputed)
+                                             instead of the default zone + node/energy pair */
 
 typedef struct {
   int32_t abi_version;          /* must be HYDRO_ABI_VERSION */
@@ -153,10 +155,12 @@ int hydro_destroy(hydro_ctx *h);
 
 /* Measurement helper (bench.py): run ncycles cycles WITHOUT CUDA graphs on the context stream,
    bracketing each kernel class with CUDA events, and report mean device milliseconds:
-   out_ms[0] per cycle-kernel launch (fused kernel, or zone+node+energy of one domain when split),
-   out_ms[1] halo exchange per cycle, out_ms[2] dt finalize per cycle, out_ms[3] whole cycle.
+   out_ms[0] cycle kernels of one domain (zone + node/energy stage by default; the one fused
+   kernel with HYDRO_FLAG_ONE_KERNEL; zone+node+energy with HYDRO_FLAG_SPLIT),
+   out_ms[1] halo exchange per cycle, out_ms[2] dt finalize per cycle, out_ms[3] whole cycle,
+   out_ms[4] zone stage and out_ms[5] node/energy stage of one domain (default path, else 0).
    Advances the state like hydro_step.  Collective. */
-int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[4]);
+int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]);
 
 /* Number of kernels of this library launched per cycle on this rank (bench.py gpu_launches). */
 int hydro_kernels_per_cycle(const hydro_ctx *h);

@@ -43,7 +43,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     nccl = _nccl_dir()
     nvcc = os.environ.get("NVCC", "nvcc")
-    cmd = [nvcc, "-shared", "-Xcompiler", "-fPIC", "-O3", "-std=c++17", "-lineinfo", *ARCH,
+    extra = os.environ.get("HYDRO_NVCC_FLAGS", "").split()
+    cmd = [nvcc, "-shared", *extra, "-Xcompiler", "-fPIC", "-O3", "-std=c++17", "-lineinfo", *ARCH,
            "-Xptxas", "-v" if verbose else "-O3",
            "-I", os.path.join(ROOT, "include"), "-I", os.path.join(nccl, "include"),
            "-o", LIB + ".tmp", *sources(),

@@ -1,23 +1,12 @@
-// kernel_fused.cu -- the whole cycle S1-S8 (+ the block part of S9's dt min) in ONE kernel.
+// kernel_node.cu -- node/energy stage of the two-kernel cycle (S5 face form, S7, S8).
 //
-// Blocking.  A block owns a TX x TY column of zones of one domain and marches it
-// through a z-chunk [k0, k1) ("2.5-D" blocking).  Node planes stream in through TMA
-// (cp.async.bulk.tensor, one 36x15 box per field, mbarrier completion) into a 3-slot ring two
-// planes ahead of use, so HBM latency is off the critical path.  Per zone plane p, separated by
-// __syncthreads:
-//   X  half-step positions x_p = x + dt/2 u of node plane p+1 (S1) into a 2-plane ring;
-//   Z  zone stage on the (TX+2) x (TY+2) zones of plane p, i.e. the tile plus a one-zone ring
-//      that is recomputed redundantly instead of exchanged: faces, corner vectors, V, DV,
-//      predictor, EOS, q, P, dt_z^2 (S2-S4, S6);
-//   G  per-face force vectors g_f = (P_below - P_above) A_f / 4 of each zone's three low faces
-//      (the face form of S5: the node force sum_z P_z B_z,l regrouped by faces);
-//   N  node stage on node plane p: F = sum of the 12 incident g_f, m_p, a, reflecting walls,
-//      u', u_half, x' (S7), written to HBM;
-//   E  energy stage on zone plane p-1: W = P sum_l B_l.u_half_l in face form
-//      (psi_f = A_f . sum of u_half over the face), e' = e - dt W / m (S8), written to HBM.
-// HBM traffic per zone-cycle is the algorithmic minimum (read x,u,m,e; write x,u,e) plus the
-// re-read of the tile's halo columns; every intermediate lives in registers or shared memory.
-// No tensor cores: nothing here is a dense contraction (BASELINE.json north_star).
+// Same 2.5-D blocking as kernel_fused.cu (TMA node-plane ring, one-zone ring per tile), but the
+// zone physics is not recomputed: P of every zone of the tile and its ring comes from HBM, written
+// by the zone stage (kernel_zone.cu).  Per plane the ring zones only form their three low face
+// vectors (x-low, y-low, z-low) from the half-step positions; then
+//   G  g_f = (P_below - P_above) A_f / 4 per face (the face form of S5),
+//   N  node plane p: F = sum of 12 incident g_f, m_p, a, walls, u', u_half, x' (S7),
+//   E  zone plane p-1: W = P sum_l B_l.u_half_l in face form, e' = e - dt W / m (S8).
 #include <algorithm>
 #include <cmath>
 
@@ -31,7 +20,7 @@ namespace hydro {
 namespace {
 
 template <int TX, int TY>
-struct Tile {
+struct NTile {
   static constexpr int TXT = TX + 2, TYT = TY + 2;  // zone-stage tile (owned + 1 ring)
   static constexpr int NZT = TXT * TYT;
   static constexpr int NTHR = (NZT + 31) / 32 * 32;
@@ -57,10 +46,10 @@ struct Tile {
 };
 
 template <int TX, int TY>
-__global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
-    k_cycle_fused(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st,
+__global__ void __launch_bounds__(NTile<TX, TY>::NTHR, 1)
+    k_node_energy(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st,
                   int KZ) {
-  using T = Tile<TX, TY>;
+  using T = NTile<TX, TY>;
   // dynamic shared memory only (no static __shared__ in this kernel), so the window starts
   // 1024-byte aligned and every TMA destination (multiples of 128 B) is aligned
   extern __shared__ __align__(1024) double sm[];
@@ -147,7 +136,6 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
   double axp = 0, ayp = 0, azp = 0, bxp = 0, byp = 0, bzp = 0;  // x-low / y-low faces, plane p-1
   double Sx = 0, Sy = 0, Sz = 0, Msum_prev = 0;                   // in-plane node sums, plane p-1
   double psi_zlow = 0.0;
-  double dt2min = INFINITY;
 
   const int64_t gxz = d.lo[0] + li, gyz = d.lo[1] + lj;
   const bool zone_xy_exists = active && li <= n0 && lj <= n1 && gxz >= 0 && gxz < d.N[0] &&
@@ -169,13 +157,14 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
   double *eng = d.en + (int64_t)(lj + 1) * d.zsx + (li + 1);
   const int64_t nrow = (int64_t)(lj + 1) * d.nsx + (li + 1);
   const int64_t gz_lo = -d.lo[2], gz_hi = d.N[2] - d.lo[2];  // plane q exists iff in [lo, hi)
-  const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
 
   // zone mass / energy of plane q (prefetched one plane ahead into registers)
-  double m_nx = 0.0, e_nx = 0.0;
+  const double *Pg = d.P + (int64_t)(lj + 1) * d.zsx + (li + 1);
+  double m_nx = 0.0, e_nx = 0.0, P_nx = 0.0;
   if (zone_xy_exists && q0 >= gz_lo && q0 < gz_hi) {
     m_nx = mg[(int64_t)(q0 + 1) * zsxy];
     e_nx = eg[(int64_t)(q0 + 1) * zsxy];
+    P_nx = Pg[(int64_t)(q0 + 1) * zsxy];
   }
 
   wait_plane(q0);
@@ -184,96 +173,35 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
   for (int p = k0 - 1; p <= k1; ++p) {
     // ---------------------------------------------------------------- X
     if (t == 0 && p + 2 <= k1 + 1) issue(p + 2);  // slot of plane p-1, free since step p-1
-    const double m = m_nx, e = e_nx;
+    const double m = m_nx, e = e_nx, P_cur = P_nx;
     const bool exists = zone_xy_exists && p >= gz_lo && p < gz_hi;
     {
       const int q = p + 1;
       const bool ok = q <= k1 && zone_xy_exists && q >= gz_lo && q < gz_hi;
       m_nx = ok ? mg[(int64_t)(q + 1) * zsxy] : 0.0;
       e_nx = ok ? eg[(int64_t)(q + 1) * zsxy] : 0.0;
+      P_nx = ok ? Pg[(int64_t)(q + 1) * zsxy] : 0.0;
     }
     wait_plane(p + 1);
     form_xp(p + 1);
     MS[t] = m;
     __syncthreads();
-    // ---------------------------------------------------------------- Z
-    const double *Ra = raw(p), *Rb = raw(p + 1);
-    double P, im;
+    // ---------------------------------------------------------------- Z (faces only)
+    const double *Ra = raw(p);
+    const double P = P_cur;
+    const double im = exists ? frcp(m) : 0.0;
     double ax0, ay0, az0, bx0, by0, bz0, cx0, cy0, cz0;
     {
       const double *Xa = XP + (p & 1) * 3 * T::RS, *Xb = XP + ((p + 1) & 1) * 3 * T::RS;
       double X[8], Y[8], Z[8];
 #pragma unroll
-      for (int l = 0; l < 8; ++l) {
+      for (int l = 0; l < 7; ++l) {  // corners 0..6 (corner 7 is on no low face)
         const int n = nidx + ((l >> 1) & 1) * T::BXN + (l & 1);
         ld3((l >> 2) ? Xb : Xa, T::RS, n, X[l], Y[l], Z[l]);
       }
-      double fx[6], fy[6], fz[6];
-#pragma unroll
-      for (int a = 0; a < 2; ++a) HYDRO_FACE(X, Y, Z, a + 6, a, a + 4, a + 2, fx[a], fy[a], fz[a]);
-#pragma unroll
-      for (int b = 0; b < 2; ++b)
-        HYDRO_FACE(X, Y, Z, 5 + 2 * b, 2 * b, 1 + 2 * b, 2 * b + 4, fx[2 + b], fy[2 + b], fz[2 + b]);
-#pragma unroll
-      for (int c = 0; c < 2; ++c)
-        HYDRO_FACE(X, Y, Z, 3 + 4 * c, 4 * c, 2 + 4 * c, 1 + 4 * c, fx[4 + c], fy[4 + c], fz[4 + c]);
-      double V8 = 0.0, DV8 = 0.0;
-#pragma unroll
-      for (int l = 0; l < 8; ++l) {
-        const int a = l & 1, b = (l >> 1) & 1, c = (l >> 2) & 1;
-        const double sx = (a ? fx[1] : -fx[0]) + (b ? fx[3] : -fx[2]) + (c ? fx[5] : -fx[4]);
-        const double sy = (a ? fy[1] : -fy[0]) + (b ? fy[3] : -fy[2]) + (c ? fy[5] : -fy[4]);
-        const double sz = (a ? fz[1] : -fz[0]) + (b ? fz[3] : -fz[2]) + (c ? fz[5] : -fz[4]);
-        if (l > 0) V8 += (X[l] - X[0]) * sx + (Y[l] - Y[0]) * sy + (Z[l] - Z[0]) * sz;
-        const double *Us = (c ? Rb : Ra) + 3 * T::RS;
-        const int n = nidx + b * T::BXN + a;
-        DV8 += Us[n] * sx + Us[T::RS + n] * sy + Us[2 * T::RS + n] * sz;
-      }
-      const double V = V8 * (1.0 / 24.0);
-      const double DV = 0.125 * DV8;
-      double a2 = fx[0] * fx[0] + fy[0] * fy[0] + fz[0] * fz[0];
-#pragma unroll
-      for (int f = 1; f < 6; ++f) {
-        const double v = fx[f] * fx[f] + fy[f] * fy[f] + fz[f] * fz[f];
-        a2 = v > a2 ? v : a2;
-      }
-      // S2-S4 and S6 with branch-free reciprocals; L = 2V/sqrt(a2) enters only through
-      // s = L(-D) = -2 DV/sqrt(a2) and through dt^2 = min(cfl^2 L^2/sigma^2, c_vol^2/D^2).
-      const double iV = frcp(V);
-      im = frcp(m);
-      const double rho = m * iV;
-      const double epos = e > 0.0 ? e : 0.0;
-      const double ep = e - (hh * (ph.gm1 * rho) * epos) * DV * im;
-      const double eppos = ep > 0.0 ? ep : 0.0;
-      const double pr = ph.gm1 * rho * eppos;
-      const double c2 = ph.ggm1 * eppos;
-      double qr = 0.0;
-      if (DV < 0.0) {  // S4: compression only (sign(D) = sign(DV) for V > 0)
-        const double c = fsqrt(c2);
-        const double s = -2.0 * DV * frsqrt(a2);
-        qr = s * (ph.q_quad * s + ph.q_lin * c);
-      }
-      // dt_z^2 = V^2 min(4 cfl^2 / (a2 sigma^2), c_vol^2 / DV^2): one reciprocal; denominators
-      // below 1e-290 mean dt_z^2 > 1e270 V^2 (never the minimum), taken as +inf.
-      const double V2 = V * V;
-      const double n1c = cfl4 * V2, d1c = (c2 + 2.0 * qr) * a2;
-      const double n2c = cv2 * V2, d2c = DV * DV;
-      const bool ok1 = d1c > 1e-290, ok2 = d2c > 1e-290;
-      const bool pick1 = ok1 && (!ok2 || n1c * d2c < n2c * d1c);
-      const double num = pick1 ? n1c : n2c, den = pick1 ? d1c : d2c;
-      const double dt2 = (ok1 || ok2) ? num * frcp(den) : INFINITY;
-      P = exists ? pr + rho * qr : 0.0;
-      if (exists && p >= k0 && p < k1 && zone_owned_xy) {
-        if (!(V > 0.0) || !isfinite(P)) {
-          const int64_t gzi = ((d.lo[2] + p) * d.N[1] + gyz) * (int64_t)d.N[0] + gxz;
-          flag_error_zone(st, (V > 0.0) ? ERR_NONFINITE : ERR_TANGLED, gzi);
-        }
-        dt2min = dt2 < dt2min ? dt2 : dt2min;
-      }
-      im = exists ? im : 0.0;
-      ax0 = fx[0]; ay0 = fy[0]; az0 = fz[0];  // x-low face
-      bx0 = fx[2]; by0 = fy[2]; bz0 = fz[2];  // y-low face
-      cx0 = fx[4]; cy0 = fy[4]; cz0 = fz[4];  // z-low face (node plane p)
+      HYDRO_FACE(X, Y, Z, 6, 0, 4, 2, ax0, ay0, az0);  // x-low (AX_0)
+      HYDRO_FACE(X, Y, Z, 5, 0, 1, 4, bx0, by0, bz0);  // y-low (AY_0)
+      HYDRO_FACE(X, Y, Z, 3, 0, 2, 1, cx0, cy0, cz0);  // z-low (AZ_0, node plane p)
       PS[t] = P;
     }
     __syncthreads();
@@ -380,16 +308,10 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
     axp = ax0; ayp = ay0; azp = az0;
     bxp = bx0; byp = by0; bzp = bz0;
   }
-  // S9 (block part): dt = sqrt(min dt^2), one atomicMin per block.
-  block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);
 }
 
-#ifndef HYDRO_FTY
-#define HYDRO_FTY 12
-#endif
-constexpr int FTX = 32, FTY = HYDRO_FTY;
+constexpr int NTX = 32, NTY = 12;
 
-// z-chunk length: minimise (waves of blocks) x (planes per block incl. the 2 warm-up planes).
 int choose_kz(int tiles, int n2, int sms) {
   int best = n2, best_cost = 1 << 30;
   for (int kz = 4; kz <= n2; ++kz) {
@@ -406,24 +328,23 @@ int choose_kz(int tiles, int n2, int sms) {
 
 }  // namespace
 
-size_t fused_smem_bytes() { return Tile<FTX, FTY>::BYTES; }
-int fused_box_y() { return Tile<FTX, FTY>::BYN; }
+int node_box_y() { return NTile<NTX, NTY>::BYN; }
 
-void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
+void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                         cudaStream_t s) {
-  using T = Tile<FTX, FTY>;
+  using T = NTile<NTX, NTY>;
   static int sms = 0;
   if (!sms) {
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaFuncSetAttribute(k_cycle_fused<FTX, FTY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(k_node_energy<NTX, NTY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)T::BYTES);
   }
-  const int tx = (d.n[0] + FTX - 1) / FTX, ty = (d.n[1] + FTY - 1) / FTY;
+  const int tx = (d.n[0] + NTX - 1) / NTX, ty = (d.n[1] + NTY - 1) / NTY;
   const int KZ = choose_kz(tx * ty, d.n[2], sms);
   dim3 grid(tx, ty, (d.n[2] + KZ - 1) / KZ);
-  k_cycle_fused<FTX, FTY><<<grid, T::NTHR, T::BYTES, s>>>(maps, d, ph, st, KZ);
+  k_node_energy<NTX, NTY><<<grid, T::NTHR, T::BYTES, s>>>(maps, d, ph, st, KZ);
 }
 
 }  // namespace hydro

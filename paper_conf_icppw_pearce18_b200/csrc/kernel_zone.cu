@@ -1,0 +1,231 @@
+// kernel_zone.cu -- zone stage of the two-kernel cycle (S1-S4, S6): P and dt_z for every zone.
+//
+// Every zone of the domain and its ghost ring (local [-1, n] per axis) is computed exactly once:
+// half-step positions x_p = x + dt/2 u (S1), face and corner vectors, V, DV (S2), the energy
+// predictor and EOS (S3), the artificial viscosity and P = p + q (S4), and dt_z (S6, owned zones
+// only, reduced per block and combined with one atomicMin).  P is written to HBM (8 B/zone) for
+// the node/energy kernel (kernel_node.cu).  A 32x8 block marches a z-chunk; node planes stream in
+// by TMA into a 3-slot ring one plane ahead of use, x_p is formed once per node into a 3-slot
+// ring, and a single __syncthreads per plane orders the rings.  No redundant compute: this is the
+// point of the split versus the one-kernel variant (kernel_fused.cu), which recomputes a zone
+// ring per tile.
+#include <algorithm>
+#include <cmath>
+
+#include "fastmath.cuh"
+#include "kernels.h"
+#include "tma.cuh"
+#include "zone_physics.cuh"
+
+namespace hydro {
+
+namespace {
+
+constexpr int ZBX = 32, ZBY = 8;                       // zones per block (x, y)
+constexpr int ZNX = ZONE_BOX_X, ZNY = ZBY + 1;         // TMA node box (x padded to 16 B)
+constexpr int ZNN = ZNX * ZNY;
+constexpr int ZRS = (ZNN + 15) / 16 * 16;              // stride of one node array (128 B)
+constexpr int ZOFF_RAW = 0;                            // [3 slots][6 fields][ZRS]
+constexpr int ZOFF_XP = ZOFF_RAW + 18 * ZRS;           // [3 slots][3][ZRS]
+constexpr int ZOFF_RED = ZOFF_XP + 9 * ZRS;            // [32]
+constexpr int ZOFF_BAR = ZOFF_RED + 32;                // 3 mbarriers
+constexpr int ZTOTAL = ZOFF_BAR + 4;
+constexpr size_t ZBYTES = ZTOTAL * sizeof(double);
+static_assert(ZNX >= ZBX + 1, "zone-kernel TMA box too narrow");
+
+__global__ void __launch_bounds__(ZBX *ZBY, 2)
+    k_zone_stage(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st,
+                 int KZ) {
+  extern __shared__ __align__(1024) double sm[];
+  double *RAW = sm + ZOFF_RAW, *XP = sm + ZOFF_XP;
+  uint64_t *bar = reinterpret_cast<uint64_t *>(sm + ZOFF_BAR);
+  if ((st->halted | st->done) != 0u) return;
+
+  const int t = threadIdx.x;
+  const int tx = t % ZBX, ty = t / ZBX;
+  const int n0 = d.n[0], n1 = d.n[1], n2 = d.n[2];
+  // this block's zones: local [zi0, zi0+32) x [zj0, zj0+8) x [zk0, zk1), inside [-1, n]
+  const int zi0 = -1 + blockIdx.x * ZBX, zj0 = -1 + blockIdx.y * ZBY;
+  const int zk0 = -1 + blockIdx.z * KZ;
+  const int zk1 = min(zk0 + KZ, n2 + 1);
+  const int li = zi0 + tx, lj = zj0 + ty;
+  const double dt = st->dt;
+  const double hh = 0.5 * dt;
+
+  // node plane q (local) -> slot (q - zk0) % 3; storage coordinates of the box origin
+  auto issue = [&](int q) {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    const int s = (q - zk0) % 3;
+    double *dst = RAW + s * 6 * ZRS;
+    mbar_expect_tx(&bar[s], 6u * ZNN * sizeof(double));
+#pragma unroll
+    for (int f = 0; f < 6; ++f) tma_load_3d(dst + f * ZRS, &maps.m[f], &bar[s], zi0 + 1, zj0 + 1, q + 1);
+  };
+  auto wait_plane = [&](int q) {
+    const int u = q - zk0;
+    mbar_wait(&bar[u % 3], (uint32_t)((u / 3) & 1));
+  };
+  auto form_xp = [&](int q) {
+    const double *R = RAW + ((q - zk0) % 3) * 6 * ZRS;
+    double *X = XP + ((q - zk0) % 3) * 3 * ZRS;
+    for (int n = t; n < ZNN; n += ZBX * ZBY) {
+      X[n] = fma(hh, R[3 * ZRS + n], R[n]);
+      X[ZRS + n] = fma(hh, R[4 * ZRS + n], R[ZRS + n]);
+      X[2 * ZRS + n] = fma(hh, R[5 * ZRS + n], R[2 * ZRS + n]);
+    }
+  };
+
+  if (t == 0) {
+    if (smem_u32(sm) & 127u) __trap();
+    for (int s = 0; s < 3; ++s) mbar_init(&bar[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    issue(zk0);
+    issue(zk0 + 1);
+  }
+  __syncthreads();
+  wait_plane(zk0);
+  form_xp(zk0);
+
+  const bool in_xy = li <= n0 && lj <= n1;
+  const int64_t gx = d.lo[0] + li, gy = d.lo[1] + lj;
+  const bool exists_xy = in_xy && gx >= 0 && gx < d.N[0] && gy >= 0 && gy < d.N[1];
+  const bool owned_xy = li >= 0 && lj >= 0 && li < n0 && lj < n1;
+  const int nidx = ty * ZNX + tx;
+  const int64_t zrow = (int64_t)(lj + 1) * d.zsx + (li + 1);
+  const int64_t gz_lo = -d.lo[2], gz_hi = d.N[2] - d.lo[2];
+  const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
+  double dt2min = INFINITY;
+
+  double m_nx = 0.0, e_nx = 0.0;
+  if (exists_xy && zk0 >= gz_lo && zk0 < gz_hi) {
+    m_nx = d.m[(int64_t)(zk0 + 1) * d.zsxy + zrow];
+    e_nx = d.e[(int64_t)(zk0 + 1) * d.zsxy + zrow];
+  }
+
+  for (int p = zk0; p < zk1; ++p) {
+    const double m = m_nx, e = e_nx;
+    const bool exists = exists_xy && p >= gz_lo && p < gz_hi;
+    {
+      const int q = p + 1;
+      const bool ok = q < zk1 && exists_xy && q >= gz_lo && q < gz_hi;
+      m_nx = ok ? d.m[(int64_t)(q + 1) * d.zsxy + zrow] : 0.0;
+      e_nx = ok ? d.e[(int64_t)(q + 1) * d.zsxy + zrow] : 0.0;
+    }
+    wait_plane(p + 1);
+    form_xp(p + 1);
+    __syncthreads();
+    if (t == 0 && p + 2 <= zk1) issue(p + 2);  // into the slot of plane p-1 (no longer read)
+    const double *Xa = XP + ((p - zk0) % 3) * 3 * ZRS, *Xb = XP + ((p + 1 - zk0) % 3) * 3 * ZRS;
+    const double *Ua = RAW + ((p - zk0) % 3) * 6 * ZRS + 3 * ZRS;
+    const double *Ub = RAW + ((p + 1 - zk0) % 3) * 6 * ZRS + 3 * ZRS;
+    double X[8], Y[8], Z[8];
+#pragma unroll
+    for (int l = 0; l < 8; ++l) {
+      const double *S = (l >> 2) ? Xb : Xa;
+      const int n = nidx + ((l >> 1) & 1) * ZNX + (l & 1);
+      X[l] = S[n];
+      Y[l] = S[ZRS + n];
+      Z[l] = S[2 * ZRS + n];
+    }
+    double fx[6], fy[6], fz[6];
+#pragma unroll
+    for (int a = 0; a < 2; ++a) HYDRO_FACE(X, Y, Z, a + 6, a, a + 4, a + 2, fx[a], fy[a], fz[a]);
+#pragma unroll
+    for (int b = 0; b < 2; ++b)
+      HYDRO_FACE(X, Y, Z, 5 + 2 * b, 2 * b, 1 + 2 * b, 2 * b + 4, fx[2 + b], fy[2 + b], fz[2 + b]);
+#pragma unroll
+    for (int c = 0; c < 2; ++c)
+      HYDRO_FACE(X, Y, Z, 3 + 4 * c, 4 * c, 2 + 4 * c, 1 + 4 * c, fx[4 + c], fy[4 + c], fz[4 + c]);
+    double V8 = 0.0, DV8 = 0.0;
+#pragma unroll
+    for (int l = 0; l < 8; ++l) {
+      const int a = l & 1, b = (l >> 1) & 1, c = (l >> 2) & 1;
+      const double sx = (a ? fx[1] : -fx[0]) + (b ? fx[3] : -fx[2]) + (c ? fx[5] : -fx[4]);
+      const double sy = (a ? fy[1] : -fy[0]) + (b ? fy[3] : -fy[2]) + (c ? fy[5] : -fy[4]);
+      const double sz = (a ? fz[1] : -fz[0]) + (b ? fz[3] : -fz[2]) + (c ? fz[5] : -fz[4]);
+      if (l > 0) V8 += (X[l] - X[0]) * sx + (Y[l] - Y[0]) * sy + (Z[l] - Z[0]) * sz;
+      const double *Us = c ? Ub : Ua;
+      const int n = nidx + b * ZNX + a;
+      DV8 += Us[n] * sx + Us[ZRS + n] * sy + Us[2 * ZRS + n] * sz;
+    }
+    const double V = V8 * (1.0 / 24.0);
+    const double DV = 0.125 * DV8;
+    double a2 = fx[0] * fx[0] + fy[0] * fy[0] + fz[0] * fz[0];
+#pragma unroll
+    for (int f = 1; f < 6; ++f) {
+      const double v = fx[f] * fx[f] + fy[f] * fy[f] + fz[f] * fz[f];
+      a2 = v > a2 ? v : a2;
+    }
+    // S2-S4, S6 (see kernel_fused.cu for the algebra): L = 2V/sqrt(a2) enters through
+    // s = -2 DV/sqrt(a2) and dt^2 = V^2 min(4 cfl^2/(a2 sigma^2), c_vol^2/DV^2).
+    const double iV = frcp(V);
+    const double im = frcp(m);
+    const double rho = m * iV;
+    const double epos = e > 0.0 ? e : 0.0;
+    const double ep = e - (hh * (ph.gm1 * rho) * epos) * DV * im;
+    const double eppos = ep > 0.0 ? ep : 0.0;
+    const double pr = ph.gm1 * rho * eppos;
+    const double c2 = ph.ggm1 * eppos;
+    double qr = 0.0;
+    if (DV < 0.0) {
+      const double c = fsqrt(c2);
+      const double s = -2.0 * DV * frsqrt(a2);
+      qr = s * (ph.q_quad * s + ph.q_lin * c);
+    }
+    const double P = exists ? pr + rho * qr : 0.0;
+    if (in_xy) d.P[(int64_t)(p + 1) * d.zsxy + zrow] = P;
+    if (exists && owned_xy && p >= 0 && p < n2) {
+      const double V2 = V * V;
+      const double n1c = cfl4 * V2, d1c = (c2 + 2.0 * qr) * a2;
+      const double n2c = cv2 * V2, d2c = DV * DV;
+      const bool ok1 = d1c > 1e-290, ok2 = d2c > 1e-290;
+      const bool pick1 = ok1 && (!ok2 || n1c * d2c < n2c * d1c);
+      const double num = pick1 ? n1c : n2c, den = pick1 ? d1c : d2c;
+      const double dt2 = (ok1 || ok2) ? num * frcp(den) : INFINITY;
+      dt2min = dt2 < dt2min ? dt2 : dt2min;
+      if (!(V > 0.0) || !isfinite(P)) {
+        const int64_t gzi = ((d.lo[2] + p) * d.N[1] + gy) * (int64_t)d.N[0] + gx;
+        flag_error_zone(st, (V > 0.0) ? ERR_NONFINITE : ERR_TANGLED, gzi);
+      }
+    }
+  }
+  block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + ZOFF_RED);
+}
+
+int choose_kz_zone(int tiles, int nplanes, int slots) {
+  int best = nplanes, best_cost = 1 << 30;
+  for (int kz = 4; kz <= nplanes; ++kz) {
+    const int chunks = (nplanes + kz - 1) / kz;
+    const int waves = (tiles * chunks + slots - 1) / slots;
+    const int cost = waves * (kz + 1);
+    if (cost < best_cost) {
+      best_cost = cost;
+      best = kz;
+    }
+  }
+  return best;
+}
+
+}  // namespace
+
+int zone_box_y() { return ZNY; }
+
+void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
+                       cudaStream_t s) {
+  static int slots = 0;
+  if (!slots) {
+    int dev = 0, sms = 0, per_sm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaFuncSetAttribute(k_zone_stage, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ZBYTES);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_zone_stage, ZBX * ZBY, ZBYTES);
+    slots = sms * std::max(per_sm, 1);
+  }
+  const int nz_x = d.n[0] + 2, nz_y = d.n[1] + 2, nz_z = d.n[2] + 2;  // zones incl. ghost ring
+  const int tx = (nz_x + ZBX - 1) / ZBX, ty = (nz_y + ZBY - 1) / ZBY;
+  const int KZ = choose_kz_zone(tx * ty, nz_z, slots);
+  dim3 grid(tx, ty, (nz_z + KZ - 1) / KZ);
+  k_zone_stage<<<grid, ZBX * ZBY, ZBYTES, s>>>(maps, d, ph, st, KZ);
+}
+
+}  // namespace hydro

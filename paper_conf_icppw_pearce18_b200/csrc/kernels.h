@@ -6,6 +6,7 @@
 #include "device.cuh"
 
 #define FUSED_BOX_X 36  // TMA node box width (TX + 3 = 35 rounded up to a 16-byte row)
+#define ZONE_BOX_X 34   // zone-stage node box width (33 rounded up to a 16-byte row)
 
 namespace hydro {
 
@@ -41,6 +42,14 @@ void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, 
                         cudaStream_t s);
 size_t fused_smem_bytes();
 int fused_box_y();
+
+// Two-kernel cycle (default path): zone stage (P, dt) then node/energy stage.
+void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
+                       cudaStream_t s);
+void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
+                        cudaStream_t s);
+int zone_box_y();
+int node_box_y();
 
 // End of cycle: S9 dt / time update and error latch.
 void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s);

@@ -30,7 +30,8 @@ struct LocalDom {
   void *mem = nullptr;
   size_t bytes = 0;
   DomView view[2];  // parity p reads view[p].x and writes view[p].xn
-  NodeMaps maps[2]; // TMA descriptors of view[p]'s current node arrays
+  NodeMaps maps[2];  // TMA descriptors of view[p]'s current node arrays, fused/node box
+  NodeMaps zmaps[2]; // same arrays, zone-stage box
 };
 
 }  // namespace
@@ -50,6 +51,7 @@ struct hydro_ctx {
   cudaGraphExec_t graph[2] = {nullptr, nullptr};
   int parity = 0;
   bool split = false;
+  bool one_kernel = false;
   bool use_graph = true;
   int failed = 0;
   Comm *comm = nullptr;
@@ -124,17 +126,23 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
   for (int par = 0; par < 2; ++par) {
     const double *arr[6] = {D.view[par].x, D.view[par].y, D.view[par].z,
                             D.view[par].u, D.view[par].v, D.view[par].w};
-    for (int f = 0; f < 6; ++f) {
-      cuuint64_t dims[3] = {(cuuint64_t)nsx, (cuuint64_t)(n1 + 3), (cuuint64_t)(n2 + 3)};
-      cuuint64_t strides[2] = {(cuuint64_t)(nsx * sizeof(double)),
-                               (cuuint64_t)(nsxy * sizeof(double))};
-      cuuint32_t box[3] = {FUSED_BOX_X, (cuuint32_t)fused_box_y(), 1};
-      cuuint32_t es[3] = {1, 1, 1};
-      CUresult r = encode(&D.maps[par].m[f], CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3,
-                          const_cast<double *>(arr[f]), dims, strides, box, es,
-                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                          CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-      if (r != CUDA_SUCCESS) return set_err(h, HYDRO_ECUDA, "cuTensorMapEncodeTiled failed");
+    for (int kind = 0; kind < 2; ++kind) {
+      if (kind == 0 && fused_box_y() != node_box_y())
+        return set_err(h, HYDRO_EINVAL, "fused and node kernels must share a TMA box");
+      for (int f = 0; f < 6; ++f) {
+        cuuint64_t dims[3] = {(cuuint64_t)nsx, (cuuint64_t)(n1 + 3), (cuuint64_t)(n2 + 3)};
+        cuuint64_t strides[2] = {(cuuint64_t)(nsx * sizeof(double)),
+                                 (cuuint64_t)(nsxy * sizeof(double))};
+        cuuint32_t box[3] = {kind ? (cuuint32_t)ZONE_BOX_X : (cuuint32_t)FUSED_BOX_X,
+                             kind ? (cuuint32_t)zone_box_y() : (cuuint32_t)fused_box_y(), 1};
+        cuuint32_t es[3] = {1, 1, 1};
+        CUresult r = encode(kind ? &D.zmaps[par].m[f] : &D.maps[par].m[f],
+                            CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double *>(arr[f]),
+                            dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                            CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) return set_err(h, HYDRO_ECUDA, "cuTensorMapEncodeTiled failed");
+      }
     }
   }
   return HYDRO_OK;
@@ -220,12 +228,19 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
     }
     for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
     for (LocalDom &D : h->doms) launch_energy_split(D.view[par], h->ph, h->st, s);
-  } else {
+  } else if (h->one_kernel) {
     for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, s);
     if (h->comm) {
       int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
     }
+  } else {
+    for (LocalDom &D : h->doms) launch_zone_stage(D.view[par], D.zmaps[par], h->ph, h->st, s);
+    if (h->comm) {
+      int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
+      if (rc) return set_err(h, rc, "dt allreduce failed");
+    }
+    for (LocalDom &D : h->doms) launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, s);
   }
   launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
   if (h->comm) {
@@ -363,6 +378,7 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
   h->ph.t_stop = cfg->t_stop;
   h->ph.reflect_mask = cfg->reflect_mask;
   h->split = (cfg->flags & HYDRO_FLAG_SPLIT) != 0;
+  h->one_kernel = !h->split && (cfg->flags & HYDRO_FLAG_ONE_KERNEL) != 0;
   h->use_graph = (cfg->flags & HYDRO_FLAG_NO_GRAPH) == 0;
   h->device = cfg->device;
   *out = nullptr;
@@ -610,32 +626,38 @@ int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, 
 int hydro_kernels_per_cycle(const hydro_ctx *h) {
   if (!h) return HYDRO_EINVAL;
   const int nd = (int)h->doms.size();
-  int k = h->split ? 3 * nd : nd;   // cycle kernels
+  int k = (h->split ? 3 : (h->one_kernel ? 1 : 2)) * nd;  // cycle kernels
   if (h->n_local_pairs > 0) k += 1;  // intra-GPU halo copy
   k += 1;                            // finalize
   if (h->comm) k += comm_kernels_per_cycle(h->comm);
   return k;
 }
 
-int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[4]) {
+int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
   if (!h || ncycles <= 0 || !out_ms) return set_err(h, HYDRO_EINVAL, "bad argument");
   if (h->failed) return set_err(h, HYDRO_ESTATE, "context failed earlier");
   CK(cudaSetDevice(h->device));
   cudaStream_t s = h->stream;
   cudaEvent_t ev[5];
   for (int i = 0; i < 5; ++i) CK(cudaEventCreate(&ev[i]));
-  double acc[4] = {0, 0, 0, 0};
+  double acc[6] = {0, 0, 0, 0, 0, 0};
   for (int32_t c = 0; c < ncycles; ++c) {
     const int par = h->parity;
     CK(cudaEventRecord(ev[0], s));
+    CK(cudaEventRecord(ev[4], s));
     if (h->split) {
       for (LocalDom &D : h->doms) launch_zone_split(D.view[par], h->ph, h->st, s);
       if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
       for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
       for (LocalDom &D : h->doms) launch_energy_split(D.view[par], h->ph, h->st, s);
-    } else {
+    } else if (h->one_kernel) {
       for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, s);
       if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
+    } else {
+      for (LocalDom &D : h->doms) launch_zone_stage(D.view[par], D.zmaps[par], h->ph, h->st, s);
+      if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
+      CK(cudaEventRecord(ev[4], s));
+      for (LocalDom &D : h->doms) launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, s);
     }
     CK(cudaEventRecord(ev[1], s));
     launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
@@ -650,6 +672,13 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[4]) {
     CK(cudaEventElapsedTime(&cc, ev[2], ev[3]));
     CK(cudaEventElapsedTime(&d, ev[0], ev[3]));
     acc[0] += a; acc[1] += b; acc[2] += cc; acc[3] += d;
+    if (!h->split && !h->one_kernel) {
+      float z, n;
+      CK(cudaEventElapsedTime(&z, ev[0], ev[4]));
+      CK(cudaEventElapsedTime(&n, ev[4], ev[1]));
+      acc[4] += z;
+      acc[5] += n;
+    }
     h->parity ^= 1;
   }
   for (int i = 0; i < 5; ++i) cudaEventDestroy(ev[i]);
@@ -658,6 +687,8 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[4]) {
   out_ms[1] = acc[1] / ncycles;
   out_ms[2] = acc[2] / ncycles;
   out_ms[3] = acc[3] / ncycles;
+  out_ms[4] = acc[4] / ncycles / nd;
+  out_ms[5] = acc[5] / ncycles / nd;
   hydro_info info;
   const int status = read_info(h, &info, s);
   if (status < 0 && status != HYDRO_ECUDA) h->failed = status;

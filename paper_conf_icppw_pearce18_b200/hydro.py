@@ -24,6 +24,7 @@ ALL_FIELDS = NODE_FIELDS + ZONE_FIELDS
 ABI_VERSION = 1
 FLAG_NO_GRAPH = 1 << 0
 FLAG_SPLIT = 1 << 1
+FLAG_ONE_KERNEL = 1 << 2
 
 STATUS = {0: "ok", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENCCL", -5: "ETANGLED",
           -6: "ENONFINITE", -7: "EDTMIN", -8: "ESTATE"}
@@ -130,7 +131,8 @@ class HydroConfig:
     rank: int = 0
     nranks: int = 1
     device: int = 0
-    split: bool = False           # HYDRO_FLAG_SPLIT: 3-kernel pipeline instead of fused
+    path: str = "two"             # "two" (zone + node/energy kernels), "one" (one fused kernel),
+                                  # "split" (plain 3-kernel pipeline, HYDRO_FLAG_SPLIT)
     graph: bool = True            # CUDA graphs (HYDRO_FLAG_NO_GRAPH when False)
 
 
@@ -177,7 +179,8 @@ def _cfg_struct(cfg: HydroConfig, keep: list, comm_id: Optional[bytes] = None) -
         buf = C.create_string_buffer(comm_id, 128)
         keep.append(buf)
         c.comm_id = C.cast(buf, C.c_void_p)
-    c.flags = (0 if cfg.graph else FLAG_NO_GRAPH) | (FLAG_SPLIT if cfg.split else 0)
+    c.flags = ((0 if cfg.graph else FLAG_NO_GRAPH) | (FLAG_SPLIT if cfg.path == "split" else 0)
+               | (FLAG_ONE_KERNEL if cfg.path == "one" else 0))
     return c
 
 
@@ -273,12 +276,12 @@ class Hydro:
 
     def time_kernels(self, ncycles: int) -> dict:
         """hydro_time_kernels: per-kernel-class mean device ms (no graphs, CUDA events)."""
-        out = (C.c_double * 4)()
+        out = (C.c_double * 6)()
         rc = self._L.hydro_time_kernels(self._h, int(ncycles), out)
         if rc in (-3, -4, -1, -8):
             raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
         return {"cycle_kernel_ms": out[0], "halo_ms": out[1], "finalize_ms": out[2],
-                "cycle_ms": out[3]}
+                "cycle_ms": out[3], "zone_stage_ms": out[4], "node_stage_ms": out[5]}
 
     def kernels_per_cycle(self) -> int:
         return int(self._L.hydro_kernels_per_cycle(self._h))

@@ -18,7 +18,7 @@ from tests.helpers import rel_err, total_energy, user_state
 pytestmark = pytest.mark.gpu
 
 FIELDS = ("x", "y", "z", "u", "v", "w", "rho", "e", "p", "q", "c", "vol", "mass")
-PATHS = [False, True]  # split=False: fused default path; split=True: 3-kernel pipeline
+PATHS = ["two", "one", "split"]  # zone+node/energy kernels (default), one fused kernel, plain split
 
 
 def run_gpu(ncycles, **kw):
@@ -42,61 +42,61 @@ def ocfg(gk):
     return OracleConfig(**{k: v for k, v in gk.items() if k in keys})
 
 
-@pytest.mark.parametrize("split", PATHS)
-def test_sedov32_one_and_hundred_cycles(split):
+@pytest.mark.parametrize("path", PATHS)
+def test_sedov32_one_and_hundred_cycles(path):
     kw = dict(n=(32, 32, 32))
     for nc, tol in ((1, 1e-12), (100, 1e-10)):
         fo, io = oracle.run(ocfg(kw), nc)
-        fg, ig = run_gpu(nc, split=split, **kw)
+        fg, ig = run_gpu(nc, path=path, **kw)
         assert ig["status"] == 0 and ig["cycle"] == nc
         compare(fg, fo, tol)
         assert ig["t"] == pytest.approx(io["t"], rel=tol)
         assert ig["dt"] == pytest.approx(io["dt"], rel=tol)
 
 
-@pytest.mark.parametrize("split", PATHS)
+@pytest.mark.parametrize("path", PATHS)
 @pytest.mark.parametrize("seed", [1, 2, 3])
-def test_jittered16(seed, split):
+def test_jittered16(seed, path):
     n = (16, 16, 16)
     kw = dict(n=n, init="user", user=jittered_state(n, seed))
     for nc, tol in ((1, 1e-12), (100, 1e-10)):
         fo, io = oracle.run(ocfg(kw), nc)
-        fg, ig = run_gpu(nc, split=split, **kw)
+        fg, ig = run_gpu(nc, path=path, **kw)
         assert ig["status"] == 0
         compare(fg, fo, tol)
         assert ig["dt"] == pytest.approx(io["dt"], rel=tol)
 
 
-@pytest.mark.parametrize("split", PATHS)
-def test_ragged_mesh_several_tiles(split):
+@pytest.mark.parametrize("path", PATHS)
+def test_ragged_mesh_several_tiles(path):
     n = (77, 37, 21)  # not a multiple of any tile size; x spans several warps
     kw = dict(n=n, init="user", user=jittered_state(n, 4))
     fo, _ = oracle.run(ocfg(kw), 10)
-    fg, ig = run_gpu(10, split=split, **kw)
+    fg, ig = run_gpu(10, path=path, **kw)
     assert ig["status"] == 0
     compare(fg, fo, 1e-11)
 
 
-@pytest.mark.parametrize("split", PATHS)
-def test_multi_domain_on_one_gpu(split):
+@pytest.mark.parametrize("path", PATHS)
+def test_multi_domain_on_one_gpu(path):
     n = (24, 20, 18)
     cuts = [[0, 5, 13, 24], [0, 1, 20], [0, 9, 10, 18]]
     kw = dict(n=n, ndom=(3, 2, 3), cuts=cuts, init="user", user=jittered_state(n, 7))
     fo, _ = oracle.run(ocfg(kw), 25)
-    fg, ig = run_gpu(25, split=split, **kw)
+    fg, ig = run_gpu(25, path=path, **kw)
     assert ig["status"] == 0
     compare(fg, fo, 1e-10)
     single = dict(kw)
     single.update(ndom=(1, 1, 1), cuts=None)
-    fs, _ = run_gpu(25, split=split, **single)
+    fs, _ = run_gpu(25, path=path, **single)
     for k in FIELDS:  # same kernels on the same inputs: bitwise
         assert np.array_equal(fs[k], fg[k]), k
 
 
-@pytest.mark.parametrize("split", PATHS)
-def test_energy_conserved_and_mass_constant(split):
+@pytest.mark.parametrize("path", PATHS)
+def test_energy_conserved_and_mass_constant(path):
     kw = dict(n=(24, 24, 24))
-    with Hydro(HydroConfig(split=split, **kw)) as h:
+    with Hydro(HydroConfig(path=path, **kw)) as h:
         f0 = h.fields()
         h.step(100)
         f = h.fields()
@@ -105,11 +105,11 @@ def test_energy_conserved_and_mass_constant(split):
     assert np.array_equal(f["mass"], f0["mass"])
 
 
-@pytest.mark.parametrize("split", PATHS)
-def test_uniform_rest_bitwise(split):
+@pytest.mark.parametrize("path", PATHS)
+def test_uniform_rest_bitwise(path):
     n = (8, 8, 8)
     s = user_state(n, extent=(1.0, 1.0, 1.0))
-    with Hydro(HydroConfig(n=n, extent=(1.0, 1.0, 1.0), init="user", user=s, split=split)) as h:
+    with Hydro(HydroConfig(n=n, extent=(1.0, 1.0, 1.0), init="user", user=s, path=path)) as h:
         f0 = h.fields()
         h.step(50)
         f = h.fields()
