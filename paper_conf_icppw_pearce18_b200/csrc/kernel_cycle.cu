@@ -1,22 +1,21 @@
-// kernel_fused.cu -- the whole cycle S1-S8 (+ the block part of S9's dt min) in ONE kernel.
+// kernel_cycle.cu -- the node/energy side of the cycle (S5 face form, S7, S8), either with the
+// zone physics recomputed in the same kernel (FUSED: the whole cycle S1-S8 in ONE kernel) or
+// with P read from HBM as written by the zone-stage kernel (kernel_zone.cu).
 //
 // Blocking.  A block owns a TX x TY column of zones of one domain and marches it
-// through a z-chunk [k0, k1) ("2.5-D" blocking).  Node planes stream in through TMA
-// (cp.async.bulk.tensor, one 36x15 box per field, mbarrier completion) into a 3-slot ring two
-// planes ahead of use, so HBM latency is off the critical path.  Per zone plane p, separated by
-// __syncthreads:
-//   X  half-step positions x_p = x + dt/2 u of node plane p+1 (S1) into a 2-plane ring;
-//   Z  zone stage on the (TX+2) x (TY+2) zones of plane p, i.e. the tile plus a one-zone ring
-//      that is recomputed redundantly instead of exchanged: faces, corner vectors, V, DV,
-//      predictor, EOS, q, P, dt_z^2 (S2-S4, S6);
-//   G  per-face force vectors g_f = (P_below - P_above) A_f / 4 of each zone's three low faces
-//      (the face form of S5: the node force sum_z P_z B_z,l regrouped by faces);
-//   N  node stage on node plane p: F = sum of the 12 incident g_f, m_p, a, reflecting walls,
-//      u', u_half, x' (S7), written to HBM;
-//   E  energy stage on zone plane p-1: W = P sum_l B_l.u_half_l in face form
-//      (psi_f = A_f . sum of u_half over the face), e' = e - dt W / m (S8), written to HBM.
-// HBM traffic per zone-cycle is the algorithmic minimum (read x,u,m,e; write x,u,e) plus the
-// re-read of the tile's halo columns; every intermediate lives in registers or shared memory.
+// through a z-chunk [k0, k1) (2.5-D blocking).  Thread (tx, ty) stands for zone and node
+// (i0-1+tx, j0-1+ty): the tile plus a one-zone ring, which is recomputed instead of exchanged.
+// Node planes stream in through TMA (one box per field, mbarrier completion) into a 3-slot ring
+// two planes ahead of use.  Per zone plane p, separated by __syncthreads:
+//   X  own node of plane p+1: x_p = x + dt/2 u (S1), kept in registers and shared;
+//   Z  zone plane p: FUSED -- faces, corner vectors, V, DV, predictor, EOS, q, P, dt_z^2
+//      (S2-S4, S6); otherwise P comes from HBM and only the three low faces are formed;
+//   G  per-face force vectors g_f = (P_below - P_above) A_f / 4 of each zone's low faces (S5 in
+//      face form: sum_z P_z B_z,l regrouped by faces);
+//   N  node plane p: F = sum of the 12 incident g_f (4 own, 5 read), m_p, a, reflecting walls,
+//      u', u_half, x' (S7), written to HBM; u_half and its two-plane sum are shared;
+//   E  zone plane p-1: psi_f = A_f . (sum of u_half over the face), W = P/8 sum_f +-psi_f,
+//      e' = e - dt W / m (S8), written to HBM.
 // No tensor cores: nothing here is a dense contraction (BASELINE.json north_star).
 #include <algorithm>
 #include <cmath>
@@ -31,7 +30,7 @@ namespace hydro {
 namespace {
 
 template <int TX, int TY>
-struct Tile {
+struct CTile {
   static constexpr int TXT = TX + 2, TYT = TY + 2;  // zone-stage tile (owned + 1 ring)
   static constexpr int NZT = TXT * TYT;
   static constexpr int NTHR = (NZT + 31) / 32 * 32;
@@ -39,12 +38,13 @@ struct Tile {
   static constexpr int BXN = FUSED_BOX_X, BYN = TY + 3;  // TMA node box (x padded to 16 B)
   static constexpr int NN = BXN * BYN;
   static constexpr int RS = (NN + 15) / 16 * 16;    // stride of one node array (128 B aligned)
-  // shared-memory layout, in doubles; every array is SoA so a warp's LDS.64 is conflict-free
+  // shared memory, in doubles; SoA everywhere so a warp's LDS.64 is conflict-free
   static constexpr int OFF_RAW = 0;                 // [3 slots][6 fields][RS] x,y,z,u,v,w (TMA)
   static constexpr int OFF_XP = OFF_RAW + 18 * RS;  // [2 planes][3][RS] half-step positions
   static constexpr int OFF_G = OFF_XP + 6 * RS;     // [3 vectors][3][ZS] g_x, g_y, g_z
-  static constexpr int OFF_UH = OFF_G + 9 * ZS;     // [2 planes][3][ZS] u_half
-  static constexpr int OFF_P = OFF_UH + 6 * ZS;     // [ZS] P of zone plane p
+  static constexpr int OFF_UH = OFF_G + 9 * ZS;     // [3][ZS] u_half of node plane p
+  static constexpr int OFF_VS = OFF_UH + 3 * ZS;    // [3][ZS] u_half(p-1) + u_half(p)
+  static constexpr int OFF_P = OFF_VS + 3 * ZS;     // [ZS] P of zone plane p
   static constexpr int OFF_M = OFF_P + ZS;          // [ZS] m of zone plane p
   static constexpr int OFF_PS = OFF_M + ZS;         // [2][ZS] psi of x-low, y-low faces
   static constexpr int OFF_RED = OFF_PS + 2 * ZS;   // [32] block dt reduction
@@ -56,18 +56,17 @@ struct Tile {
   static_assert(BYTES <= 227 * 1024, "shared memory");
 };
 
-template <int TX, int TY>
-__global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
-    k_cycle_fused(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st,
-                  int KZ) {
-  using T = Tile<TX, TY>;
-  // dynamic shared memory only (no static __shared__ in this kernel), so the window starts
-  // 1024-byte aligned and every TMA destination (multiples of 128 B) is aligned
+template <int TX, int TY, bool FUSED>
+__global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
+    k_cycle(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st, int KZ) {
+  using T = CTile<TX, TY>;
+  // dynamic shared memory only (no static __shared__), so the window is 1024-byte aligned
   extern __shared__ __align__(1024) double sm[];
   double *RAW = sm + T::OFF_RAW, *XP = sm + T::OFF_XP, *PS = sm + T::OFF_P, *MS = sm + T::OFF_M;
-  double *G = sm + T::OFF_G;  // g_x at [0, 3ZS), g_y at [3ZS, 6ZS), g_z at [6ZS, 9ZS)
-  double *UH = sm + T::OFF_UH, *PSX = sm + T::OFF_PS, *PSY = PSX + T::ZS;
+  double *GX = sm + T::OFF_G, *GY = GX + 3 * T::ZS, *GZ = GY + 3 * T::ZS;
+  double *UH = sm + T::OFF_UH, *VS = sm + T::OFF_VS, *PSX = sm + T::OFF_PS, *PSY = PSX + T::ZS;
   uint64_t *bar = reinterpret_cast<uint64_t *>(sm + T::OFF_BAR);
+  constexpr int ZS = T::ZS, RS = T::RS, TXT = T::TXT;
 
   const int t = threadIdx.x;
   const int i0 = blockIdx.x * TX, j0 = blockIdx.y * TY;
@@ -76,7 +75,7 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
   const int n0 = d.n[0], n1 = d.n[1], n2 = d.n[2];
   const bool active = t < T::NZT;
   const int tc = active ? t : T::NZT - 1;  // padding lanes shadow the last zone (never store)
-  const int tx = tc % T::TXT, ty = tc / T::TXT;
+  const int tx = tc % TXT, ty = tc / TXT;
   const int li = i0 - 1 + tx, lj = j0 - 1 + ty;  // local zone / node index of this thread
 
   if ((st->halted | st->done) != 0u) {  // no-op cycle: carry the state over to the next parity
@@ -105,32 +104,43 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
   auto issue = [&](int q) {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     const int u = q - q0, s = u % 3;
-    double *dst = RAW + s * 6 * T::RS;
+    double *dst = RAW + s * 6 * RS;
     mbar_expect_tx(&bar[s], 6u * T::NN * sizeof(double));
 #pragma unroll
-    for (int f = 0; f < 6; ++f) tma_load_3d(dst + f * T::RS, &maps.m[f], &bar[s], i0, j0, q + 1);
+    for (int f = 0; f < 6; ++f) tma_load_3d(dst + f * RS, &maps.m[f], &bar[s], i0, j0, q + 1);
   };
   auto wait_plane = [&](int q) {
     const int u = q - q0;
     mbar_wait(&bar[u % 3], (uint32_t)((u / 3) & 1));
   };
-  auto raw = [&](int q) { return RAW + ((q - q0) % 3) * 6 * T::RS; };
-  // X stage: half-step positions of node plane q into XP slot q&1.
-  auto form_xp = [&](int q) {
+  auto raw = [&](int q) { return RAW + ((q - q0) % 3) * 6 * RS; };
+  // X stage: half-step positions of node plane q into XP slot q&1.  Thread t forms its own
+  // node (tx, ty) -- returned in registers -- and the box's last column / row are shared out.
+  const int nidx = ty * T::BXN + tx;  // this thread's node in the node box
+  auto form_xp = [&](int q, double &px, double &py, double &pz) {
     const double *R = raw(q);
-    double *X = XP + (q & 1) * 3 * T::RS;
-    for (int n = t; n < T::NN; n += T::NTHR) {
-      X[n] = fma(hh, R[3 * T::RS + n], R[n]);
-      X[T::RS + n] = fma(hh, R[4 * T::RS + n], R[T::RS + n]);
-      X[2 * T::RS + n] = fma(hh, R[5 * T::RS + n], R[2 * T::RS + n]);
+    double *X = XP + (q & 1) * 3 * RS;
+    px = fma(hh, R[3 * RS + nidx], R[nidx]);
+    py = fma(hh, R[4 * RS + nidx], R[RS + nidx]);
+    pz = fma(hh, R[5 * RS + nidx], R[2 * RS + nidx]);
+    if (active) {
+      X[nidx] = px;
+      X[RS + nidx] = py;
+      X[2 * RS + nidx] = pz;
+    }
+    // remaining nodes of the box: column TXT (rows 0..TYT) and row TYT (columns 0..TXT-1)
+    for (int e = t; e < T::TYT + 1 + TXT; e += T::NTHR) {
+      const int n = e <= T::TYT ? e * T::BXN + TXT : T::TYT * T::BXN + (e - T::TYT - 1);
+      X[n] = fma(hh, R[3 * RS + n], R[n]);
+      X[RS + n] = fma(hh, R[4 * RS + n], R[RS + n]);
+      X[2 * RS + n] = fma(hh, R[5 * RS + n], R[2 * RS + n]);
     }
   };
-  // 3-vectors in SoA shared arrays: component k of item i at base[k*stride + i]
-  auto st3 = [](double *b, int stride, int i, double x, double y, double z) {
-    b[i] = x; b[stride + i] = y; b[2 * stride + i] = z;
+  auto st3 = [](double *b, int i, double x, double y, double z) {
+    b[i] = x; b[ZS + i] = y; b[2 * ZS + i] = z;
   };
-  auto ld3 = [](const double *b, int stride, int i, double &x, double &y, double &z) {
-    x = b[i]; y = b[stride + i]; z = b[2 * stride + i];
+  auto ld3 = [](const double *b, int i, double &x, double &y, double &z) {
+    x = b[i]; y = b[ZS + i]; z = b[2 * ZS + i];
   };
 
   if (t == 0) {
@@ -146,6 +156,7 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
   double P_prev = 0.0, im_prev = 0.0, e_prev = 0.0;
   double axp = 0, ayp = 0, azp = 0, bxp = 0, byp = 0, bzp = 0;  // x-low / y-low faces, plane p-1
   double Sx = 0, Sy = 0, Sz = 0, Msum_prev = 0;                   // in-plane node sums, plane p-1
+  double uhp = 0, vhp = 0, whp = 0;                               // own u_half of plane p-1
   double psi_zlow = 0.0;
   double dt2min = INFINITY;
 
@@ -159,54 +170,63 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
   const bool ex_x = active && tx >= 1 && tx <= TX + 1 && ty >= 1 && ty <= TY;
   const bool ex_y = active && tx >= 1 && tx <= TX && ty >= 1 && ty <= TY + 1;
   const bool ex_z = active && tx >= 1 && tx <= TX && ty >= 1 && ty <= TY;
-  const int nidx = ty * T::BXN + tx;  // this thread's node in the node box
   const uint32_t rm = ph.reflect_mask;
   const bool wall_x = (gxz == 0 && (rm & 1u)) || (gxz == d.N[0] && (rm & 2u));
   const bool wall_y = (gyz == 0 && (rm & 4u)) || (gyz == d.N[1] && (rm & 8u));
   const int64_t zsxy = d.zsxy, nsxy = d.nsxy;
-  const double *mg = d.m + (int64_t)(lj + 1) * d.zsx + (li + 1);  // + (q+1)*zsxy
-  const double *eg = d.e + (int64_t)(lj + 1) * d.zsx + (li + 1);
-  double *eng = d.en + (int64_t)(lj + 1) * d.zsx + (li + 1);
+  const int64_t zoff = (int64_t)(lj + 1) * d.zsx + (li + 1);  // + (q+1)*zsxy
   const int64_t nrow = (int64_t)(lj + 1) * d.nsx + (li + 1);
   const int64_t gz_lo = -d.lo[2], gz_hi = d.N[2] - d.lo[2];  // plane q exists iff in [lo, hi)
   const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
 
-  // zone mass / energy of plane q (prefetched one plane ahead into registers)
-  double m_nx = 0.0, e_nx = 0.0;
+  // zone mass / energy (and P when not FUSED) of plane q, prefetched one plane ahead
+  double m_nx = 0.0, e_nx = 0.0, P_nx = 0.0;
   if (zone_xy_exists && q0 >= gz_lo && q0 < gz_hi) {
-    m_nx = mg[(int64_t)(q0 + 1) * zsxy];
-    e_nx = eg[(int64_t)(q0 + 1) * zsxy];
+    m_nx = d.m[(int64_t)(q0 + 1) * zsxy + zoff];
+    e_nx = d.e[(int64_t)(q0 + 1) * zsxy + zoff];
+    if (!FUSED) P_nx = d.P[(int64_t)(q0 + 1) * zsxy + zoff];
   }
 
+  double xpa, ypa, zpa;  // own node's x_p at plane p (corner 0 of the own zone)
   wait_plane(q0);
-  form_xp(q0);
+  form_xp(q0, xpa, ypa, zpa);
 
   for (int p = k0 - 1; p <= k1; ++p) {
     // ---------------------------------------------------------------- X
     if (t == 0 && p + 2 <= k1 + 1) issue(p + 2);  // slot of plane p-1, free since step p-1
     const double m = m_nx, e = e_nx;
+    double P = FUSED ? 0.0 : P_nx;
     const bool exists = zone_xy_exists && p >= gz_lo && p < gz_hi;
     {
       const int q = p + 1;
       const bool ok = q <= k1 && zone_xy_exists && q >= gz_lo && q < gz_hi;
-      m_nx = ok ? mg[(int64_t)(q + 1) * zsxy] : 0.0;
-      e_nx = ok ? eg[(int64_t)(q + 1) * zsxy] : 0.0;
+      const int64_t zq = (int64_t)(q + 1) * zsxy + zoff;
+      m_nx = ok ? d.m[zq] : 0.0;
+      e_nx = ok ? d.e[zq] : 0.0;
+      if (!FUSED) P_nx = ok ? d.P[zq] : 0.0;
     }
     wait_plane(p + 1);
-    form_xp(p + 1);
+    double xpb, ypb, zpb;  // own node's x_p at plane p+1 (corner 4)
+    form_xp(p + 1, xpb, ypb, zpb);
     MS[t] = m;
+    if (!FUSED) PS[t] = P;
     __syncthreads();
-    // ---------------------------------------------------------------- Z
-    const double *Ra = raw(p), *Rb = raw(p + 1);
-    double P, im;
+    // ---------------------------------------------------------------- Z (+ G when not FUSED)
+    const double *Ra = raw(p);
+    const double *Xa = XP + (p & 1) * 3 * RS, *Xb = XP + ((p + 1) & 1) * 3 * RS;
+    double im;
     double ax0, ay0, az0, bx0, by0, bz0, cx0, cy0, cz0;
-    {
-      const double *Xa = XP + (p & 1) * 3 * T::RS, *Xb = XP + ((p + 1) & 1) * 3 * T::RS;
+    if (FUSED) {
+      const double *Rb = raw(p + 1);
       double X[8], Y[8], Z[8];
+      X[0] = xpa; Y[0] = ypa; Z[0] = zpa;
+      X[4] = xpb; Y[4] = ypb; Z[4] = zpb;
 #pragma unroll
       for (int l = 0; l < 8; ++l) {
+        if (l == 0 || l == 4) continue;
         const int n = nidx + ((l >> 1) & 1) * T::BXN + (l & 1);
-        ld3((l >> 2) ? Xb : Xa, T::RS, n, X[l], Y[l], Z[l]);
+        const double *S = (l >> 2) ? Xb : Xa;
+        X[l] = S[n]; Y[l] = S[RS + n]; Z[l] = S[2 * RS + n];
       }
       double fx[6], fy[6], fz[6];
 #pragma unroll
@@ -225,9 +245,9 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
         const double sy = (a ? fy[1] : -fy[0]) + (b ? fy[3] : -fy[2]) + (c ? fy[5] : -fy[4]);
         const double sz = (a ? fz[1] : -fz[0]) + (b ? fz[3] : -fz[2]) + (c ? fz[5] : -fz[4]);
         if (l > 0) V8 += (X[l] - X[0]) * sx + (Y[l] - Y[0]) * sy + (Z[l] - Z[0]) * sz;
-        const double *Us = (c ? Rb : Ra) + 3 * T::RS;
+        const double *Us = (c ? Rb : Ra) + 3 * RS;
         const int n = nidx + b * T::BXN + a;
-        DV8 += Us[n] * sx + Us[T::RS + n] * sy + Us[2 * T::RS + n] * sz;
+        DV8 += Us[n] * sx + Us[RS + n] * sy + Us[2 * RS + n] * sz;
       }
       const double V = V8 * (1.0 / 24.0);
       const double DV = 0.125 * DV8;
@@ -237,8 +257,8 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
         const double v = fx[f] * fx[f] + fy[f] * fy[f] + fz[f] * fz[f];
         a2 = v > a2 ? v : a2;
       }
-      // S2-S4 and S6 with branch-free reciprocals; L = 2V/sqrt(a2) enters only through
-      // s = L(-D) = -2 DV/sqrt(a2) and through dt^2 = min(cfl^2 L^2/sigma^2, c_vol^2/D^2).
+      // S2-S4 and S6: L = 2V/sqrt(a2) enters only through s = L(-D) = -2 DV/sqrt(a2) and
+      // dt^2 = V^2 min(4 cfl^2/(a2 sigma^2), c_vol^2/DV^2) (one reciprocal)
       const double iV = frcp(V);
       im = frcp(m);
       const double rho = m * iV;
@@ -253,77 +273,91 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
         const double s = -2.0 * DV * frsqrt(a2);
         qr = s * (ph.q_quad * s + ph.q_lin * c);
       }
-      // dt_z^2 = V^2 min(4 cfl^2 / (a2 sigma^2), c_vol^2 / DV^2): one reciprocal; denominators
-      // below 1e-290 mean dt_z^2 > 1e270 V^2 (never the minimum), taken as +inf.
-      const double V2 = V * V;
-      const double n1c = cfl4 * V2, d1c = (c2 + 2.0 * qr) * a2;
-      const double n2c = cv2 * V2, d2c = DV * DV;
-      const bool ok1 = d1c > 1e-290, ok2 = d2c > 1e-290;
-      const bool pick1 = ok1 && (!ok2 || n1c * d2c < n2c * d1c);
-      const double num = pick1 ? n1c : n2c, den = pick1 ? d1c : d2c;
-      const double dt2 = (ok1 || ok2) ? num * frcp(den) : INFINITY;
       P = exists ? pr + rho * qr : 0.0;
       if (exists && p >= k0 && p < k1 && zone_owned_xy) {
+        const double V2 = V * V;
+        const double n1c = cfl4 * V2, d1c = (c2 + 2.0 * qr) * a2;
+        const double n2c = cv2 * V2, d2c = DV * DV;
+        const bool ok1 = d1c > 1e-290, ok2 = d2c > 1e-290;  // else dt_z^2 > 1e270 V^2: +inf
+        const bool pick1 = ok1 && (!ok2 || n1c * d2c < n2c * d1c);
+        const double num = pick1 ? n1c : n2c, den = pick1 ? d1c : d2c;
+        const double dt2 = (ok1 || ok2) ? num * frcp(den) : INFINITY;
+        dt2min = dt2 < dt2min ? dt2 : dt2min;
         if (!(V > 0.0) || !isfinite(P)) {
           const int64_t gzi = ((d.lo[2] + p) * d.N[1] + gyz) * (int64_t)d.N[0] + gxz;
           flag_error_zone(st, (V > 0.0) ? ERR_NONFINITE : ERR_TANGLED, gzi);
         }
-        dt2min = dt2 < dt2min ? dt2 : dt2min;
       }
-      im = exists ? im : 0.0;
       ax0 = fx[0]; ay0 = fy[0]; az0 = fz[0];  // x-low face
       bx0 = fx[2]; by0 = fy[2]; bz0 = fz[2];  // y-low face
       cx0 = fx[4]; cy0 = fy[4]; cz0 = fz[4];  // z-low face (node plane p)
       PS[t] = P;
+      __syncthreads();
+    } else {
+      double X[7], Y[7], Z[7];  // corners 0..6 (corner 7 lies on no low face)
+      X[0] = xpa; Y[0] = ypa; Z[0] = zpa;
+      X[4] = xpb; Y[4] = ypb; Z[4] = zpb;
+#pragma unroll
+      for (int l = 1; l < 7; ++l) {
+        if (l == 4) continue;
+        const int n = nidx + ((l >> 1) & 1) * T::BXN + (l & 1);
+        const double *S = (l >> 2) ? Xb : Xa;
+        X[l] = S[n]; Y[l] = S[RS + n]; Z[l] = S[2 * RS + n];
+      }
+      HYDRO_FACE(X, Y, Z, 6, 0, 4, 2, ax0, ay0, az0);  // x-low (AX_0)
+      HYDRO_FACE(X, Y, Z, 5, 0, 1, 4, bx0, by0, bz0);  // y-low (AY_0)
+      HYDRO_FACE(X, Y, Z, 3, 0, 2, 1, cx0, cy0, cz0);  // z-low (AZ_0, node plane p)
+      im = exists ? frcp(m) : 0.0;
     }
-    __syncthreads();
+    if (FUSED) im = exists ? im : 0.0;
     // ---------------------------------------------------------------- G
-    {
-      const double gxw = (tx > 0) ? 0.125 * (PS[tc - 1] - P) : 0.0;
-      const double gyw = (ty > 0) ? 0.125 * (PS[tc - T::TXT] - P) : 0.0;
-      const double gzw = 0.125 * (P_prev - P);
-      st3(G, T::ZS, t, gxw * ax0, gxw * ay0, gxw * az0);
-      st3(G + 3 * T::ZS, T::ZS, t, gyw * bx0, gyw * by0, gyw * bz0);
-      st3(G + 6 * T::ZS, T::ZS, t, gzw * cx0, gzw * cy0, gzw * cz0);
-    }
+    const double gxw = (tx > 0) ? 0.125 * (PS[tc - 1] - P) : 0.0;
+    const double gyw = (ty > 0) ? 0.125 * (PS[tc - TXT] - P) : 0.0;
+    const double gzw = 0.125 * (P_prev - P);
+    const double gxx = gxw * ax0, gxy = gxw * ay0, gxz_ = gxw * az0;
+    const double gyx = gyw * bx0, gyy = gyw * by0, gyz_ = gyw * bz0;
+    const double gzx = gzw * cx0, gzy = gzw * cy0, gzz = gzw * cz0;
+    st3(GX, t, gxx, gxy, gxz_);
+    st3(GY, t, gyx, gyy, gyz_);
+    st3(GZ, t, gzx, gzy, gzz);
     __syncthreads();
     // ---------------------------------------------------------------- N
-    double *UHc = UH + (p & 1) * 3 * T::ZS;
-    const double *GXs = G, *GYs = G + 3 * T::ZS, *GZs = G + 6 * T::ZS;
+    double uh = 0.0, vh = 0.0, wh = 0.0;
     if (node_xy) {
-      const int tn = tc - T::TXT;  // zone (tx, ty-1)
-      double ax_, ay_, az_, bx_, by_, bz_, cx_, cy_, cz_, dx_, dy_, dz_;
-      ld3(GXs, T::ZS, tn, ax_, ay_, az_);
-      ld3(GXs, T::ZS, tc, bx_, by_, bz_);
-      ld3(GYs, T::ZS, tc - 1, cx_, cy_, cz_);
-      ld3(GYs, T::ZS, tc, dx_, dy_, dz_);
-      const double Cx = (ax_ + bx_) + (cx_ + dx_);
-      const double Cy = (ay_ + by_) + (cy_ + dy_);
-      const double Cz = (az_ + bz_) + (cz_ + dz_);
-      const double Ms = (MS[tn - 1] + MS[tn]) + (MS[tc - 1] + MS[tc]);
+      const int tn = tc - TXT;  // zone (tx, ty-1)
+      double a0, a1, a2_, b0, b1, b2;
+      ld3(GX, tn, a0, a1, a2_);      // g_x of zone (tx, ty-1)
+      ld3(GY, tc - 1, b0, b1, b2);   // g_y of zone (tx-1, ty)
+      const double Cx = (gxx + a0) + (gyx + b0);
+      const double Cy = (gxy + a1) + (gyy + b1);
+      const double Cz = (gxz_ + a2_) + (gyz_ + b2);
+      const double Ms = (MS[tn - 1] + MS[tn]) + (MS[tc - 1] + m);
       if (p >= k0) {
-        ld3(GZs, T::ZS, tn - 1, ax_, ay_, az_);
-        ld3(GZs, T::ZS, tn, bx_, by_, bz_);
-        ld3(GZs, T::ZS, tc - 1, cx_, cy_, cz_);
-        ld3(GZs, T::ZS, tc, dx_, dy_, dz_);
-        const double Fx = Sx + Cx + ((ax_ + bx_) + (cx_ + dx_));
-        const double Fy = Sy + Cy + ((ay_ + by_) + (cy_ + dy_));
-        const double Fz = Sz + Cz + ((az_ + bz_) + (cz_ + dz_));
+        double c0, c1, c2_;
+        ld3(GZ, tn - 1, a0, a1, a2_);
+        ld3(GZ, tn, b0, b1, b2);
+        ld3(GZ, tc - 1, c0, c1, c2_);
+        const double Fx = Sx + Cx + ((a0 + b0) + (c0 + gzx));
+        const double Fy = Sy + Cy + ((a1 + b1) + (c1 + gzy));
+        const double Fz = Sz + Cz + ((a2_ + b2) + (c2_ + gzz));
         const double rinv = 8.0 * frcp(Msum_prev + Ms);
         const int64_t g2 = d.lo[2] + p;
         const bool wall_z = (g2 == 0 && (rm & 16u)) || (g2 == d.N[2] && (rm & 32u));
         const double axc = wall_x ? 0.0 : Fx * rinv;
         const double ayc = wall_y ? 0.0 : Fy * rinv;
         const double azc = wall_z ? 0.0 : Fz * rinv;
-        const double u = Ra[3 * T::RS + nidx], v = Ra[4 * T::RS + nidx], w = Ra[5 * T::RS + nidx];
+        const double u = Ra[3 * RS + nidx], v = Ra[4 * RS + nidx], w = Ra[5 * RS + nidx];
         const double un = u + dt * axc, vn = v + dt * ayc, wn = w + dt * azc;
-        const double uh = (u + un) * 0.5, vh = (v + vn) * 0.5, wh = (w + wn) * 0.5;
-        st3(UHc, T::ZS, tc, uh, vh, wh);
+        uh = (u + un) * 0.5;
+        vh = (v + vn) * 0.5;
+        wh = (w + wn) * 0.5;
+        st3(UH, tc, uh, vh, wh);
+        st3(VS, tc, uhp + uh, vhp + vh, whp + wh);
         if (node_write_xy && (p < k1 || p == n2)) {
           const int64_t id = (int64_t)(p + 1) * nsxy + nrow;
           d.xn[id] = Ra[nidx] + dt * uh;
-          d.yn[id] = Ra[T::RS + nidx] + dt * vh;
-          d.zn[id] = Ra[2 * T::RS + nidx] + dt * wh;
+          d.yn[id] = Ra[RS + nidx] + dt * vh;
+          d.zn[id] = Ra[2 * RS + nidx] + dt * wh;
           d.un[id] = un;
           d.vn[id] = vn;
           d.wn[id] = wn;
@@ -334,44 +368,35 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
     }
     __syncthreads();
     // ---------------------------------------------------------------- E
-    double psi_zhigh = 0.0;
+    double psi_zhigh = 0.0, psx = 0.0, psy = 0.0;
+    const double vsx = uhp + uh, vsy = vhp + vh, vsz = whp + wh;  // own two-plane u_half sum
     if (p >= k0) {
-      const double *UHp = UH + ((p - 1) & 1) * 3 * T::ZS;
-      double a0, a1, a2_, b0, b1, b2, c0, c1, c2_, e0, e1, e2;
+      double a0, a1, a2_, b0, b1, b2, c0, c1, c2_;
       if (p >= k0 + 1) {
-        if (ex_x) {  // x-low face of zone plane p-1: nodes (tx, ty..ty+1) at planes p-1, p
-          const int t2 = tc + T::TXT;
-          ld3(UHp, T::ZS, tc, a0, a1, a2_);
-          ld3(UHp, T::ZS, t2, b0, b1, b2);
-          ld3(UHc, T::ZS, tc, c0, c1, c2_);
-          ld3(UHc, T::ZS, t2, e0, e1, e2);
-          PSX[t] = axp * ((a0 + b0) + (c0 + e0)) + ayp * ((a1 + b1) + (c1 + e1)) +
-                   azp * ((a2_ + b2) + (c2_ + e2));
+        if (ex_x) {  // x-low face of zone plane p-1: nodes (tx, ty..ty+1), planes p-1, p
+          ld3(VS, tc + TXT, a0, a1, a2_);
+          psx = axp * (vsx + a0) + ayp * (vsy + a1) + azp * (vsz + a2_);
+          PSX[t] = psx;
         }
-        if (ex_y) {  // y-low face of zone plane p-1: nodes (tx..tx+1, ty) at planes p-1, p
-          const int t2 = tc + 1;
-          ld3(UHp, T::ZS, tc, a0, a1, a2_);
-          ld3(UHp, T::ZS, t2, b0, b1, b2);
-          ld3(UHc, T::ZS, tc, c0, c1, c2_);
-          ld3(UHc, T::ZS, t2, e0, e1, e2);
-          PSY[t] = bxp * ((a0 + b0) + (c0 + e0)) + byp * ((a1 + b1) + (c1 + e1)) +
-                   bzp * ((a2_ + b2) + (c2_ + e2));
+        if (ex_y) {  // y-low face of zone plane p-1: nodes (tx..tx+1, ty), planes p-1, p
+          ld3(VS, tc + 1, a0, a1, a2_);
+          psy = bxp * (vsx + a0) + byp * (vsy + a1) + bzp * (vsz + a2_);
+          PSY[t] = psy;
         }
       }
       if (ex_z) {  // z-face at node plane p: nodes (tx..tx+1, ty..ty+1)
-        ld3(UHc, T::ZS, tc, a0, a1, a2_);
-        ld3(UHc, T::ZS, tc + 1, b0, b1, b2);
-        ld3(UHc, T::ZS, tc + T::TXT, c0, c1, c2_);
-        ld3(UHc, T::ZS, tc + T::TXT + 1, e0, e1, e2);
-        psi_zhigh = cx0 * ((a0 + b0) + (c0 + e0)) + cy0 * ((a1 + b1) + (c1 + e1)) +
-                    cz0 * ((a2_ + b2) + (c2_ + e2));
+        ld3(UH, tc + 1, a0, a1, a2_);
+        ld3(UH, tc + TXT, b0, b1, b2);
+        ld3(UH, tc + TXT + 1, c0, c1, c2_);
+        psi_zhigh = cx0 * ((uh + a0) + (b0 + c0)) + cy0 * ((vh + a1) + (b1 + c1)) +
+                    cz0 * ((wh + a2_) + (b2 + c2_));
       }
     }
     __syncthreads();
     if (p >= k0 + 1 && zone_owned_xy) {
       const double Wk = 0.125 * P_prev *
-                        (((PSX[t + 1] - PSX[t]) + (PSY[t + T::TXT] - PSY[t])) + (psi_zhigh - psi_zlow));
-      eng[(int64_t)p * zsxy] = e_prev - dt * Wk * im_prev;
+                        (((PSX[t + 1] - psx) + (PSY[t + TXT] - psy)) + (psi_zhigh - psi_zlow));
+      d.en[(int64_t)p * zsxy + zoff] = e_prev - dt * Wk * im_prev;
     }
     psi_zlow = psi_zhigh;
     P_prev = P;
@@ -379,15 +404,13 @@ __global__ void __launch_bounds__(Tile<TX, TY>::NTHR, 1)
     e_prev = e;
     axp = ax0; ayp = ay0; azp = az0;
     bxp = bx0; byp = by0; bzp = bz0;
+    uhp = uh; vhp = vh; whp = wh;
+    xpa = xpb; ypa = ypb; zpa = zpb;
   }
-  // S9 (block part): dt = sqrt(min dt^2), one atomicMin per block.
-  block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);
+  if (FUSED) block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);
 }
 
-#ifndef HYDRO_FTY
-#define HYDRO_FTY 12
-#endif
-constexpr int FTX = 32, FTY = HYDRO_FTY;
+constexpr int CTX = 32, CTY = 12;
 
 // z-chunk length: minimise (waves of blocks) x (planes per block incl. the 2 warm-up planes).
 int choose_kz(int tiles, int n2, int sms) {
@@ -404,26 +427,37 @@ int choose_kz(int tiles, int n2, int sms) {
   return std::min(best, n2);
 }
 
-}  // namespace
-
-size_t fused_smem_bytes() { return Tile<FTX, FTY>::BYTES; }
-int fused_box_y() { return Tile<FTX, FTY>::BYN; }
-
-void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                        cudaStream_t s) {
-  using T = Tile<FTX, FTY>;
+template <bool FUSED>
+void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st, cudaStream_t s) {
+  using T = CTile<CTX, CTY>;
   static int sms = 0;
   if (!sms) {
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaFuncSetAttribute(k_cycle_fused<FTX, FTY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(k_cycle<CTX, CTY, FUSED>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)T::BYTES);
   }
-  const int tx = (d.n[0] + FTX - 1) / FTX, ty = (d.n[1] + FTY - 1) / FTY;
+  const int tx = (d.n[0] + CTX - 1) / CTX, ty = (d.n[1] + CTY - 1) / CTY;
   const int KZ = choose_kz(tx * ty, d.n[2], sms);
   dim3 grid(tx, ty, (d.n[2] + KZ - 1) / KZ);
-  k_cycle_fused<FTX, FTY><<<grid, T::NTHR, T::BYTES, s>>>(maps, d, ph, st, KZ);
+  k_cycle<CTX, CTY, FUSED><<<grid, T::NTHR, T::BYTES, s>>>(maps, d, ph, st, KZ);
+}
+
+}  // namespace
+
+size_t fused_smem_bytes() { return CTile<CTX, CTY>::BYTES; }
+int fused_box_y() { return CTile<CTX, CTY>::BYN; }
+int node_box_y() { return CTile<CTX, CTY>::BYN; }
+
+void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
+                        cudaStream_t s) {
+  launch<true>(d, maps, ph, st, s);
+}
+
+void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
+                        cudaStream_t s) {
+  launch<false>(d, maps, ph, st, s);
 }
 
 }  // namespace hydro
