@@ -310,11 +310,11 @@ def main():
         kern.append(("split zone+node+energy", kt["cycle_kernel_ms"],
                      96.0 * Nn + 24.0 * Nz, None))
     rows = []
-    for name, ms, byts, flops in kern:
-        hbm = byts / (ms * 1e-3) / 1e9
-        r = {"kernel": name, "ms": ms, "alg_bytes": byts, "hbm_gbs": hbm, "hbm_frac": hbm / peak}
+    for name, kms, byts, flops in kern:
+        hbm = byts / (kms * 1e-3) / 1e9
+        r = {"kernel": name, "ms": kms, "alg_bytes": byts, "hbm_gbs": hbm, "hbm_frac": hbm / peak}
         if flops:
-            alu = flops / (ms * 1e-3)
+            alu = flops / (kms * 1e-3)
             r.update({"fp64_inst_per_s": alu, "fp64_frac": alu / fp64_peak()})
         rows.append(r)
     dom = max(rows, key=lambda r: r["ms"])
