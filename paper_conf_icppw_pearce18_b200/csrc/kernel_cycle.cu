@@ -38,21 +38,26 @@ struct CTile {
   static constexpr int BXN = FUSED_BOX_X, BYN = TY + 3;  // TMA node box (x padded to 16 B)
   static constexpr int NN = BXN * BYN;
   static constexpr int RS = (NN + 15) / 16 * 16;    // stride of one node array (128 B aligned)
+  static constexpr int ZBX = TXT, ZBY = TYT;        // TMA zone box = the zone tile
+  static constexpr int ZN = ZBX * ZBY;
+  static constexpr int ZRS = (ZN + 15) / 16 * 16;
   // shared memory, in doubles; SoA everywhere so a warp's LDS.64 is conflict-free
   static constexpr int OFF_RAW = 0;                 // [3 slots][6 fields][RS] x,y,z,u,v,w (TMA)
-  static constexpr int OFF_XP = OFF_RAW + 18 * RS;  // [2 planes][3][RS] half-step positions
+  static constexpr int OFF_ZR = OFF_RAW + 18 * RS;  // [3 slots][3 fields][ZRS] m, e, P (TMA)
+  static constexpr int OFF_XP = OFF_ZR + 9 * ZRS;   // [2 planes][3][RS] half-step positions
   static constexpr int OFF_G = OFF_XP + 6 * RS;     // [3 vectors][3][ZS] g_x, g_y, g_z
   static constexpr int OFF_UH = OFF_G + 9 * ZS;     // [3][ZS] u_half of node plane p
   static constexpr int OFF_VS = OFF_UH + 3 * ZS;    // [3][ZS] u_half(p-1) + u_half(p)
-  static constexpr int OFF_P = OFF_VS + 3 * ZS;     // [ZS] P of zone plane p
-  static constexpr int OFF_M = OFF_P + ZS;          // [ZS] m of zone plane p
-  static constexpr int OFF_PS = OFF_M + ZS;         // [2][ZS] psi of x-low, y-low faces
+  static constexpr int OFF_P = OFF_VS + 3 * ZS;     // [ZS] P of zone plane p (FUSED)
+  static constexpr int OFF_PS = OFF_P + ZS;         // [2][ZS] psi of x-low, y-low faces
   static constexpr int OFF_RED = OFF_PS + 2 * ZS;   // [32] block dt reduction
   static constexpr int OFF_BAR = OFF_RED + 32;      // 3 mbarriers
   static constexpr int TOTAL = OFF_BAR + 4;
   static constexpr size_t BYTES = sizeof(double) * TOTAL;
   static_assert(BXN >= TX + 3, "TMA box too narrow");
   static_assert(BYN <= 256 && BXN <= 256, "TMA box limit");
+  static_assert((ZBX * 8) % 16 == 0, "TMA zone box rows must be 16-byte multiples");
+  static_assert(ZRS >= ZS - 32 && ZN <= ZS, "zone tile fits the thread tile");
   static_assert(BYTES <= 227 * 1024, "shared memory");
 };
 
@@ -62,11 +67,11 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   using T = CTile<TX, TY>;
   // dynamic shared memory only (no static __shared__), so the window is 1024-byte aligned
   extern __shared__ __align__(1024) double sm[];
-  double *RAW = sm + T::OFF_RAW, *XP = sm + T::OFF_XP, *PS = sm + T::OFF_P, *MS = sm + T::OFF_M;
+  double *RAW = sm + T::OFF_RAW, *ZR = sm + T::OFF_ZR, *XP = sm + T::OFF_XP, *PSF = sm + T::OFF_P;
   double *GX = sm + T::OFF_G, *GY = GX + 3 * T::ZS, *GZ = GY + 3 * T::ZS;
   double *UH = sm + T::OFF_UH, *VS = sm + T::OFF_VS, *PSX = sm + T::OFF_PS, *PSY = PSX + T::ZS;
   uint64_t *bar = reinterpret_cast<uint64_t *>(sm + T::OFF_BAR);
-  constexpr int ZS = T::ZS, RS = T::RS, TXT = T::TXT;
+  constexpr int ZS = T::ZS, RS = T::RS, TXT = T::TXT, ZRS = T::ZRS;
 
   const int t = threadIdx.x;
   const int i0 = blockIdx.x * TX, j0 = blockIdx.y * TY;
@@ -100,20 +105,26 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   const double hh = 0.5 * dt;
   const int q0 = k0 - 1;  // first node plane of the chunk
 
-  // TMA producer: node plane q -> slot (q-q0)%3, 6 fields, one mbarrier per slot.
+  // TMA producer: node plane q and zone plane q (m, e, and P unless FUSED) -> slot (q-q0)%3,
+  // one mbarrier per slot.  Zone plane q lies between node planes q and q+1.
+  constexpr int NZF = FUSED ? 2 : 3;
   auto issue = [&](int q) {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     const int u = q - q0, s = u % 3;
     double *dst = RAW + s * 6 * RS;
-    mbar_expect_tx(&bar[s], 6u * T::NN * sizeof(double));
+    double *zdst = ZR + s * 3 * ZRS;
+    mbar_expect_tx(&bar[s], (6u * T::NN + (unsigned)NZF * T::ZN) * sizeof(double));
 #pragma unroll
     for (int f = 0; f < 6; ++f) tma_load_3d(dst + f * RS, &maps.m[f], &bar[s], i0, j0, q + 1);
+#pragma unroll
+    for (int f = 0; f < NZF; ++f) tma_load_3d(zdst + f * ZRS, &maps.z[f], &bar[s], i0, j0, q + 1);
   };
   auto wait_plane = [&](int q) {
     const int u = q - q0;
     mbar_wait(&bar[u % 3], (uint32_t)((u / 3) & 1));
   };
   auto raw = [&](int q) { return RAW + ((q - q0) % 3) * 6 * RS; };
+  auto zraw = [&](int q) { return ZR + ((q - q0) % 3) * 3 * ZRS; };
   // X stage: half-step positions of node plane q into XP slot q&1.  Thread t forms its own
   // node (tx, ty) -- returned in registers -- and the box's last column / row are shared out.
   const int nidx = ty * T::BXN + tx;  // this thread's node in the node box
@@ -179,14 +190,6 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   const int64_t gz_lo = -d.lo[2], gz_hi = d.N[2] - d.lo[2];  // plane q exists iff in [lo, hi)
   const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
 
-  // zone mass / energy (and P when not FUSED) of plane q, prefetched one plane ahead
-  double m_nx = 0.0, e_nx = 0.0, P_nx = 0.0;
-  if (zone_xy_exists && q0 >= gz_lo && q0 < gz_hi) {
-    m_nx = d.m[(int64_t)(q0 + 1) * zsxy + zoff];
-    e_nx = d.e[(int64_t)(q0 + 1) * zsxy + zoff];
-    if (!FUSED) P_nx = d.P[(int64_t)(q0 + 1) * zsxy + zoff];
-  }
-
   double xpa, ypa, zpa;  // own node's x_p at plane p (corner 0 of the own zone)
   wait_plane(q0);
   form_xp(q0, xpa, ypa, zpa);
@@ -194,22 +197,14 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   for (int p = k0 - 1; p <= k1; ++p) {
     // ---------------------------------------------------------------- X
     if (t == 0 && p + 2 <= k1 + 1) issue(p + 2);  // slot of plane p-1, free since step p-1
-    const double m = m_nx, e = e_nx;
-    double P = FUSED ? 0.0 : P_nx;
     const bool exists = zone_xy_exists && p >= gz_lo && p < gz_hi;
-    {
-      const int q = p + 1;
-      const bool ok = q <= k1 && zone_xy_exists && q >= gz_lo && q < gz_hi;
-      const int64_t zq = (int64_t)(q + 1) * zsxy + zoff;
-      m_nx = ok ? d.m[zq] : 0.0;
-      e_nx = ok ? d.e[zq] : 0.0;
-      if (!FUSED) P_nx = ok ? d.P[zq] : 0.0;
-    }
     wait_plane(p + 1);
     double xpb, ypb, zpb;  // own node's x_p at plane p+1 (corner 4)
     form_xp(p + 1, xpb, ypb, zpb);
-    MS[t] = m;
-    if (!FUSED) PS[t] = P;
+    // zone plane p (TMA): m and e are 0 on zones outside the mesh (never written), P too
+    double *MS = zraw(p), *ES = MS + ZRS, *PS = FUSED ? PSF : MS + 2 * ZRS;
+    const double m = MS[tc], e = ES[tc];
+    double P = FUSED ? 0.0 : PS[tc];
     __syncthreads();
     // ---------------------------------------------------------------- Z (+ G when not FUSED)
     const double *Ra = raw(p);
@@ -449,6 +444,8 @@ void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st
 size_t fused_smem_bytes() { return CTile<CTX, CTY>::BYTES; }
 int fused_box_y() { return CTile<CTX, CTY>::BYN; }
 int node_box_y() { return CTile<CTX, CTY>::BYN; }
+int cycle_zone_box_x() { return CTile<CTX, CTY>::ZBX; }
+int cycle_zone_box_y() { return CTile<CTX, CTY>::ZBY; }
 
 void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                         cudaStream_t s) {

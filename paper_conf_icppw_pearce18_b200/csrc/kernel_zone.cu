@@ -31,11 +31,12 @@ constexpr int ZOFF_RED = ZOFF_XP + 9 * ZRS;            // [32]
 constexpr int ZOFF_BAR = ZOFF_RED + 32;                // 3 mbarriers
 constexpr int ZTOTAL = ZOFF_BAR + 4;
 constexpr size_t ZBYTES = ZTOTAL * sizeof(double);
-static_assert(ZNX >= ZBX + 1, "zone-kernel TMA box too narrow");
+static_assert(ZNX >= ZBX + 2, "zone-kernel TMA box too narrow (33 nodes + 1 alignment shift)");
 
 __global__ void __launch_bounds__(ZBX *ZBY, 2)
     k_zone_stage(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st,
-                 int KZ) {
+                 int KZ, int zlox, int zloy, int zloz, int zhix, int zhiy, int zhiz) {
+  const int3 zlo = make_int3(zlox, zloy, zloz), zhi = make_int3(zhix, zhiy, zhiz);
   extern __shared__ __align__(1024) double sm[];
   double *RAW = sm + ZOFF_RAW, *XP = sm + ZOFF_XP;
   uint64_t *bar = reinterpret_cast<uint64_t *>(sm + ZOFF_BAR);
@@ -44,11 +45,16 @@ __global__ void __launch_bounds__(ZBX *ZBY, 2)
   const int t = threadIdx.x;
   const int tx = t % ZBX, ty = t / ZBX;
   const int n0 = d.n[0], n1 = d.n[1], n2 = d.n[2];
-  // this block's zones: local [zi0, zi0+32) x [zj0, zj0+8) x [zk0, zk1), inside [-1, n]
-  const int zi0 = -1 + blockIdx.x * ZBX, zj0 = -1 + blockIdx.y * ZBY;
-  const int zk0 = -1 + blockIdx.z * KZ;
-  const int zk1 = min(zk0 + KZ, n2 + 1);
+  // this block's zones: local [zi0, zi0+32) x [zj0, zj0+8) x [zk0, zk1) inside [zlo, zhi):
+  // the owned zones plus the ghost ring where a neighbouring domain exists (ghost zones beyond
+  // the physical boundary do not exist; their P stays 0)
+  const int zi0 = zlo.x + blockIdx.x * ZBX, zj0 = zlo.y + blockIdx.y * ZBY;
+  const int zk0 = zlo.z + blockIdx.z * KZ;
+  const int zk1 = min(zk0 + KZ, zhi.z);
   const int li = zi0 + tx, lj = zj0 + ty;
+  // TMA needs a 16-byte-aligned box start in x: start at the even storage column at or below the
+  // tile's first node column and shift the shared-memory index by xoff
+  const int xoff = (zi0 + 1) & 1, cx = zi0 + 1 - xoff;
   const double dt = st->dt;
   const double hh = 0.5 * dt;
 
@@ -59,7 +65,7 @@ __global__ void __launch_bounds__(ZBX *ZBY, 2)
     double *dst = RAW + s * 6 * ZRS;
     mbar_expect_tx(&bar[s], 6u * ZNN * sizeof(double));
 #pragma unroll
-    for (int f = 0; f < 6; ++f) tma_load_3d(dst + f * ZRS, &maps.m[f], &bar[s], zi0 + 1, zj0 + 1, q + 1);
+    for (int f = 0; f < 6; ++f) tma_load_3d(dst + f * ZRS, &maps.m[f], &bar[s], cx, zj0 + 1, q + 1);
   };
   auto wait_plane = [&](int q) {
     const int u = q - zk0;
@@ -86,11 +92,11 @@ __global__ void __launch_bounds__(ZBX *ZBY, 2)
   wait_plane(zk0);
   form_xp(zk0);
 
-  const bool in_xy = li <= n0 && lj <= n1;
+  const bool in_xy = li < zhi.x && lj < zhi.y;
   const int64_t gx = d.lo[0] + li, gy = d.lo[1] + lj;
   const bool exists_xy = in_xy && gx >= 0 && gx < d.N[0] && gy >= 0 && gy < d.N[1];
   const bool owned_xy = li >= 0 && lj >= 0 && li < n0 && lj < n1;
-  const int nidx = ty * ZNX + tx;
+  const int nidx = ty * ZNX + tx + xoff;
   const int64_t zrow = (int64_t)(lj + 1) * d.zsx + (li + 1);
   const int64_t gz_lo = -d.lo[2], gz_hi = d.N[2] - d.lo[2];
   const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
@@ -221,11 +227,17 @@ void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, D
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_zone_stage, ZBX * ZBY, ZBYTES);
     slots = sms * std::max(per_sm, 1);
   }
-  const int nz_x = d.n[0] + 2, nz_y = d.n[1] + 2, nz_z = d.n[2] + 2;  // zones incl. ghost ring
+  int lo[3], hi[3];
+  for (int a = 0; a < 3; ++a) {  // ghost ring only on sides with a neighbouring domain
+    lo[a] = d.lo[a] > 0 ? -1 : 0;
+    hi[a] = d.lo[a] + d.n[a] < d.N[a] ? d.n[a] + 1 : d.n[a];
+  }
+  const int nz_x = hi[0] - lo[0], nz_y = hi[1] - lo[1], nz_z = hi[2] - lo[2];
   const int tx = (nz_x + ZBX - 1) / ZBX, ty = (nz_y + ZBY - 1) / ZBY;
   const int KZ = choose_kz_zone(tx * ty, nz_z, slots);
   dim3 grid(tx, ty, (nz_z + KZ - 1) / KZ);
-  k_zone_stage<<<grid, ZBX * ZBY, ZBYTES, s>>>(maps, d, ph, st, KZ);
+  k_zone_stage<<<grid, ZBX * ZBY, ZBYTES, s>>>(maps, d, ph, st, KZ, lo[0], lo[1], lo[2], hi[0],
+                                               hi[1], hi[2]);
 }
 
 }  // namespace hydro

@@ -6,7 +6,7 @@
 #include "device.cuh"
 
 #define FUSED_BOX_X 36  // TMA node box width (TX + 3 = 35 rounded up to a 16-byte row)
-#define ZONE_BOX_X 34   // zone-stage node box width (33 rounded up to a 16-byte row)
+#define ZONE_BOX_X 36   // zone-stage node box width (33 + 1 alignment shift, 16-byte rows)
 
 namespace hydro {
 
@@ -32,9 +32,11 @@ void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, cudaStrea
 void launch_node_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 void launch_energy_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 
-// TMA descriptors of the six node-state arrays (x,y,z,u,v,w) of one domain and parity.
+// TMA descriptors of one domain and parity: the six node-state arrays (x,y,z,u,v,w) and the
+// zone arrays m, e, P (box = the kernel's zone tile).
 struct alignas(64) NodeMaps {
   CUtensorMap m[6];
+  CUtensorMap z[3];
 };
 
 // Fused single-kernel cycle (default path).
@@ -50,6 +52,8 @@ void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, 
                         cudaStream_t s);
 int zone_box_y();
 int node_box_y();
+int cycle_zone_box_x();  // zone-field TMA box of the cycle kernels
+int cycle_zone_box_y();
 
 // End of cycle: S9 dt / time update and error latch.
 void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s);

@@ -126,21 +126,33 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
   for (int par = 0; par < 2; ++par) {
     const double *arr[6] = {D.view[par].x, D.view[par].y, D.view[par].z,
                             D.view[par].u, D.view[par].v, D.view[par].w};
+    const double *zarr[3] = {D.view[par].m, D.view[par].e, D.view[par].P};
     for (int kind = 0; kind < 2; ++kind) {
       if (kind == 0 && fused_box_y() != node_box_y())
         return set_err(h, HYDRO_EINVAL, "fused and node kernels must share a TMA box");
-      for (int f = 0; f < 6; ++f) {
-        cuuint64_t dims[3] = {(cuuint64_t)nsx, (cuuint64_t)(n1 + 3), (cuuint64_t)(n2 + 3)};
-        cuuint64_t strides[2] = {(cuuint64_t)(nsx * sizeof(double)),
-                                 (cuuint64_t)(nsxy * sizeof(double))};
-        cuuint32_t box[3] = {kind ? (cuuint32_t)ZONE_BOX_X : (cuuint32_t)FUSED_BOX_X,
-                             kind ? (cuuint32_t)zone_box_y() : (cuuint32_t)fused_box_y(), 1};
+      NodeMaps &M = kind ? D.zmaps[par] : D.maps[par];
+      for (int f = 0; f < 9; ++f) {
+        const bool zf = f >= 6;
+        const int64_t sx = zf ? zsx : nsx, sy = zf ? (n1 + 2) : (n1 + 3);
+        const int64_t sz = zf ? (n2 + 2) : (n2 + 3), sxy = zf ? zsxy : nsxy;
+        cuuint64_t dims[3] = {(cuuint64_t)sx, (cuuint64_t)sy, (cuuint64_t)sz};
+        cuuint64_t strides[2] = {(cuuint64_t)(sx * sizeof(double)),
+                                 (cuuint64_t)(sxy * sizeof(double))};
+        cuuint32_t box[3];
+        if (zf) {
+          box[0] = (cuuint32_t)cycle_zone_box_x();
+          box[1] = (cuuint32_t)cycle_zone_box_y();
+        } else {
+          box[0] = kind ? (cuuint32_t)ZONE_BOX_X : (cuuint32_t)FUSED_BOX_X;
+          box[1] = kind ? (cuuint32_t)zone_box_y() : (cuuint32_t)fused_box_y();
+        }
+        box[2] = 1;
         cuuint32_t es[3] = {1, 1, 1};
-        CUresult r = encode(kind ? &D.zmaps[par].m[f] : &D.maps[par].m[f],
-                            CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double *>(arr[f]),
-                            dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                            CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        CUtensorMap *dst = zf ? &M.z[f - 6] : &M.m[f];
+        CUresult r = encode(dst, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3,
+                            const_cast<double *>(zf ? zarr[f - 6] : arr[f]), dims, strides, box,
+                            es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
         if (r != CUDA_SUCCESS) return set_err(h, HYDRO_ECUDA, "cuTensorMapEncodeTiled failed");
       }
     }
