@@ -147,11 +147,22 @@ def fp64_peak():
     return 1.708e13
 
 
-# Executed fp64 pipe instructions (DADD+DMUL+DFMA, thread level) per owned zone and DRAM bytes
-# per owned zone of each kernel at 128^3, from ncu (profiles/r01_*.txt).  The
-# zone stage has no redundant work, so its executed count is the algorithmic count.
-FP64_PER_ZONE = {"k_zone_stage": 0.0, "k_node_energy": 0.0, "k_cycle_fused": 516.0}
-TRAFFIC_PER_ZONE = {}
+def kernel_counters():
+    """Per-kernel ncu counters at 128^3 (profiles/kernel_counters.json, written by
+    tools/ncu_summary.py from an `ncu --set full` capture): DRAM bytes per owned
+    zone and executed fp64 pipe instructions (DADD+DMUL+DFMA, thread level) per owned zone.  The
+    zone stage computes every zone exactly once, so its executed count is the algorithmic count;
+    the tile-ring kernels recompute a ring and have no algorithmic fp64 figure here."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "kernel_counters.json")) as f:
+            return json.load(f)["kernels"]
+    except Exception:
+        return {}
+
+
+KC = kernel_counters()
+FP64_PER_ZONE = {"k_zone_stage": KC.get("k_zone_stage", {}).get("fp64_inst_per_zone")}
+TRAFFIC_PER_ZONE = {k: v.get("dram_bytes_per_zone") for k, v in KC.items()}
 
 
 def oracle_baseline(kw, budget_s=12.0):
@@ -299,13 +310,12 @@ def main():
     peak, peak_kind = measured_peak_hbm()
     kern = []
     if args.path == "two":
+        zf = FP64_PER_ZONE.get("k_zone_stage")
         kern.append(("k_zone_stage", kt["zone_stage_ms"], 48.0 * Nn + 24.0 * Nz,
-                     FP64_PER_ZONE["k_zone_stage"] * Nz))
-        kern.append(("k_node_energy", kt["node_stage_ms"], 96.0 * Nn + 32.0 * Nz,
-                     FP64_PER_ZONE["k_node_energy"] * Nz))
+                     zf * Nz if zf else None))
+        kern.append(("k_node_energy", kt["node_stage_ms"], 96.0 * Nn + 32.0 * Nz, None))
     elif args.path == "one":
-        kern.append(("k_cycle_fused", kt["cycle_kernel_ms"], 96.0 * Nn + 24.0 * Nz,
-                     FP64_PER_ZONE["k_cycle_fused"] * Nz))
+        kern.append(("k_cycle_fused", kt["cycle_kernel_ms"], 96.0 * Nn + 24.0 * Nz, None))
     else:
         kern.append(("split zone+node+energy", kt["cycle_kernel_ms"],
                      96.0 * Nn + 24.0 * Nz, None))
@@ -324,7 +334,10 @@ def main():
             "peak": fp64_peak() / 1e12 if alu_bound else peak,
             "unit": "T fp64-inst/s" if alu_bound else "GB/s",
             "frac": dom["fp64_frac"] if alu_bound else dom["hbm_frac"],
-            "traffic": TRAFFIC_PER_ZONE.get(dom["kernel"], 0) * Nz or None,
+            "traffic": (TRAFFIC_PER_ZONE[dom["kernel"]] * Nz
+                        if TRAFFIC_PER_ZONE.get(dom["kernel"]) else None),
+            "traffic_source": "ncu dram__bytes_read+write per zone at 128^3 "
+                              "(profiles/kernel_counters.json) x this launch's zones",
             "peak_source": ("measured DFMA rate (profiles/r01_fp64_peak.txt)" if alu_bound
                             else f"{peak_kind} MEASURED_PEAKS.json hbm_gbs"),
             "kernel": dom["kernel"], "kernel_ms": dom["ms"],

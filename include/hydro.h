@@ -174,6 +174,13 @@ int hydro_kernels_per_cycle(const hydro_ctx *h);
    layout tests. */
 int hydro_layout_export(const hydro_config *cfg, int64_t *buf, size_t *len);
 
+/* Inter-rank halo plan of cfg->rank (host-only; what the communicator will send and receive):
+   words [nsend, nrecv, then per message (sends first, each list in global pair order)
+   pair, peer rank, count of doubles, dst domain, src domain, direction].  Every rank enumerates
+   the messages between two ranks in the same order, which is what makes the grouped NCCL
+   send/recv match.  Returns HYDRO_EINVAL if cfg is invalid or buf is too small. */
+int hydro_comm_plan_export(const hydro_config *cfg, int64_t *buf, size_t *len);
+
 /* Hierarchical decomposition (Fig. 10a,b): split n into ngpu near-cubic
    blocks (minimum total interface area; x split last, L587), then each block into dpg slabs along
    y ("a single dimension").  Writes ndom[3], cuts (cuts[a] must hold n[a]+1 entries) and

@@ -4,8 +4,8 @@ The compute path is the CUDA library ``libhydro_b200.so`` (include/hydro.h); ``h
 thin binding and ``inputs`` the seeded synthetic input generators.  Importing the package does
 not load the library; constructing ``Hydro`` does, and fails loudly if it is missing.
 """
-from .hydro import (ALL_FIELDS, Hydro, HydroConfig, HydroError, decompose_hierarchical,  # noqa
-                    layout_export, load_library, weighted_slabs)
+from .hydro import (ALL_FIELDS, Hydro, HydroConfig, HydroError, comm_plan_export,  # noqa
+                    decompose_hierarchical, layout_export, load_library, weighted_slabs)
 
 __all__ = ["Hydro", "HydroConfig", "HydroError", "layout_export", "decompose_hierarchical",
-           "weighted_slabs", "load_library", "ALL_FIELDS"]
+           "weighted_slabs", "load_library", "ALL_FIELDS", "comm_plan_export"]

@@ -85,29 +85,29 @@ int comm_create(Comm **out, const hydro_config *cfg, const Layout &L,
     *err = "ncclCommInitRank failed";
     return HYDRO_ENCCL;
   }
-  for (const HaloPair &P : remote) {
-    SlabDesc d;
-    for (int a = 0; a < 3; ++a) {
-      d.nlo[a] = P.nlo[a]; d.nhi[a] = P.nhi[a]; d.zlo[a] = P.zlo[a]; d.zhi[a] = P.zhi[a];
-    }
-    int64_t nn = 1, nz = 1;
-    for (int a = 0; a < 3; ++a) {
-      nn *= P.nhi[a] - P.nlo[a];
-      nz *= P.zhi[a] - P.zlo[a];
-    }
-    d.count = 6 * nn + nz;
-    if (slot_of_dom[P.src] >= 0) {  // we own the source: send
-      d.slot = slot_of_dom[P.src];
-      d.peer = L.dom[P.dst].rank;
-      d.offset = c->send_total;
-      c->send_total += d.count;
-      c->sends.push_back(d);
-    } else {  // we own the destination: receive
-      d.slot = slot_of_dom[P.dst];
-      d.peer = L.dom[P.src].rank;
-      d.offset = c->recv_total;
-      c->recv_total += d.count;
-      c->recvs.push_back(d);
+  std::vector<PlanEntry> snd, rcv;
+  comm_plan(L, cfg->rank, &snd, &rcv);
+  (void)remote;
+  for (int dir = 0; dir < 2; ++dir) {
+    for (const PlanEntry &e : dir ? rcv : snd) {
+      const HaloPair &P = L.pairs[e.pair];
+      SlabDesc d;
+      for (int a = 0; a < 3; ++a) {
+        d.nlo[a] = P.nlo[a]; d.nhi[a] = P.nhi[a]; d.zlo[a] = P.zlo[a]; d.zhi[a] = P.zhi[a];
+      }
+      d.count = e.count;
+      d.peer = e.peer;
+      if (dir == 0) {  // we own the source: send
+        d.slot = slot_of_dom[P.src];
+        d.offset = c->send_total;
+        c->send_total += d.count;
+        c->sends.push_back(d);
+      } else {         // we own the destination: receive
+        d.slot = slot_of_dom[P.dst];
+        d.offset = c->recv_total;
+        c->recv_total += d.count;
+        c->recvs.push_back(d);
+      }
     }
   }
   auto ck = [&](cudaError_t e) {

@@ -164,6 +164,24 @@ std::vector<int64_t> layout_serialise(const Layout &L) {
   return w;
 }
 
+void comm_plan(const Layout &L, int32_t rank, std::vector<PlanEntry> *sends,
+               std::vector<PlanEntry> *recvs) {
+  sends->clear();
+  recvs->clear();
+  for (size_t i = 0; i < L.pairs.size(); ++i) {
+    const HaloPair &P = L.pairs[i];
+    const int32_t rd = L.dom[P.dst].rank, rs = L.dom[P.src].rank;
+    if (rd == rs) continue;  // same rank: intra-GPU copy kernel
+    int64_t nn = 1, nz = 1;
+    for (int a = 0; a < 3; ++a) {
+      nn *= P.nhi[a] - P.nlo[a];
+      nz *= P.zhi[a] - P.zlo[a];
+    }
+    if (rs == rank) sends->push_back(PlanEntry{(int32_t)i, rd, 6 * nn + nz});
+    if (rd == rank) recvs->push_back(PlanEntry{(int32_t)i, rs, 6 * nn + nz});
+  }
+}
+
 }  // namespace hydro
 
 using namespace hydro;
@@ -177,6 +195,26 @@ int hydro_layout_export(const hydro_config *cfg, int64_t *buf, size_t *len) {
   const int rc = layout_build(cfg, &L, &err);
   if (rc != HYDRO_OK) return rc;
   std::vector<int64_t> w = layout_serialise(L);
+  const size_t cap = *len;
+  *len = w.size();
+  if (buf && cap >= w.size()) std::copy(w.begin(), w.end(), buf);
+  return (buf && cap < w.size()) ? HYDRO_EINVAL : HYDRO_OK;
+}
+
+int hydro_comm_plan_export(const hydro_config *cfg, int64_t *buf, size_t *len) {
+  if (!len) return HYDRO_EINVAL;
+  Layout L;
+  std::string err;
+  const int rc = layout_build(cfg, &L, &err);
+  if (rc != HYDRO_OK) return rc;
+  std::vector<PlanEntry> snd, rcv;
+  comm_plan(L, cfg->rank, &snd, &rcv);
+  std::vector<int64_t> w{(int64_t)snd.size(), (int64_t)rcv.size()};
+  for (const auto *v : {&snd, &rcv})
+    for (const PlanEntry &e : *v) {
+      const HaloPair &P = L.pairs[e.pair];
+      w.insert(w.end(), {e.pair, e.peer, e.count, P.dst, P.src, P.dir});
+    }
   const size_t cap = *len;
   *len = w.size();
   if (buf && cap >= w.size()) std::copy(w.begin(), w.end(), buf);

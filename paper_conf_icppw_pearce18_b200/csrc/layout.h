@@ -49,4 +49,15 @@ std::vector<int32_t> lpt_assign(const std::vector<int64_t> &cost, int32_t nranks
 // Serialisation used by hydro_layout_export.
 std::vector<int64_t> layout_serialise(const Layout &L);
 
+// Inter-rank halo plan of one rank: the slabs it sends (it owns the source domain) and receives
+// (it owns the destination domain), in global pair order so that both ends of every rank pair
+// enumerate their messages identically (NCCL send/recv match in issue order).
+struct PlanEntry {
+  int32_t pair;   // index into Layout::pairs
+  int32_t peer;   // remote rank
+  int64_t count;  // doubles: 6 node fields over the node slab + e over the zone slab
+};
+void comm_plan(const Layout &L, int32_t rank, std::vector<PlanEntry> *sends,
+               std::vector<PlanEntry> *recvs);
+
 }  // namespace hydro

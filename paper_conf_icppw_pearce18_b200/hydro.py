@@ -87,6 +87,8 @@ def load_library(path: str = LIB_PATH) -> C.CDLL:
                                                C.POINTER(C.c_int32),
                                                C.POINTER(C.POINTER(C.c_int64)),
                                                C.POINTER(C.c_int32)]
+    L.hydro_comm_plan_export.argtypes = [C.POINTER(HydroConfigC), C.POINTER(C.c_int64),
+                                         C.POINTER(C.c_size_t)]
     L.hydro_weighted_slabs.argtypes = [C.c_int64, C.c_int32, C.POINTER(C.c_double),
                                        C.POINTER(C.c_int64)]
     L.hydro_comm_unique_id.argtypes = [C.c_void_p]
@@ -196,6 +198,23 @@ def layout_export(cfg: HydroConfig) -> np.ndarray:
     if rc != 0:
         raise HydroError(rc, L.hydro_last_error(None).decode())
     return buf
+
+
+def comm_plan_export(cfg: HydroConfig):
+    """hydro_comm_plan_export -> (sends, recvs), lists of (pair, peer, count, dst, src, dir)."""
+    L = load_library()
+    keep: list = []
+    c = _cfg_struct(cfg, keep)
+    n = C.c_size_t(0)
+    L.hydro_comm_plan_export(C.byref(c), None, C.byref(n))
+    buf = np.zeros(max(n.value, 2), dtype=np.int64)
+    rc = L.hydro_comm_plan_export(C.byref(c), buf.ctypes.data_as(C.POINTER(C.c_int64)),
+                                  C.byref(n))
+    if rc != 0:
+        raise HydroError(rc, "comm_plan_export")
+    ns, nr = int(buf[0]), int(buf[1])
+    ent = buf[2:].reshape(-1, 6).tolist() if ns + nr else []
+    return [tuple(e) for e in ent[:ns]], [tuple(e) for e in ent[ns:ns + nr]]
 
 
 def decompose_hierarchical(n: Sequence[int], ngpu: int, dpg: int):

@@ -1,0 +1,48 @@
+"""Summarise an ncu --set full report into per-kernel counters used by bench.py's roofline:
+DRAM bytes and executed fp64 (DADD/DMUL/DFMA) thread instructions per launch, per owned zone.
+
+    python tools/ncu_summary.py report.ncu-rep ZONES > profiles/kernel_counters.json
+"""
+import csv
+import json
+import subprocess
+import sys
+
+rep, zones = sys.argv[1], float(sys.argv[2])
+raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
+                     text=True).stdout.splitlines()
+rows = list(csv.reader(raw))
+hdr = rows[0]
+out = {}
+for vals in rows[2:]:
+    d = dict(zip(hdr, vals))
+    name = d["Kernel Name"]
+    key = "k_zone_stage" if "k_zone_stage" in name else (
+        "k_cycle_fused" if "k_cycle<" in name and ", 1>" in name else (
+            "k_node_energy" if "k_cycle<" in name else name.split("(")[0]))
+    if key in out:
+        continue
+    def f(k):
+        try:
+            return float(d[k].replace(",", ""))
+        except (KeyError, ValueError):
+            return float("nan")
+    rd, wr = f("dram__bytes_read.sum"), f("dram__bytes_write.sum")
+    unit = 1e6  # ncu reports Mbyte
+    regex = "k_zone_stage" if key == "k_zone_stage" else "k_cycle"
+    fp = subprocess.run([sys.executable, "tools/ncu_fp64_count.py", rep, regex],
+                        capture_output=True, text=True).stdout.split()
+    fp64 = float(fp[1]) if len(fp) > 1 else float("nan")
+    out[key] = {
+        "duration_us": f("gpu__time_duration.sum"),
+        "dram_bytes": (rd + wr) * unit, "dram_read_bytes": rd * unit, "dram_write_bytes": wr * unit,
+        "dram_bytes_per_zone": (rd + wr) * unit / zones,
+        "fp64_inst": fp64, "fp64_inst_per_zone": fp64 / zones,
+        "fp64_pipe_pct": f("sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active"),
+        "issue_active": f("smsp__issue_active.avg.per_cycle_active"),
+        "warps_active": f("sm__warps_active.avg.per_cycle_active"),
+        "registers": f("launch__registers_per_thread"),
+        "warp_inst": f("smsp__inst_executed.sum"),
+    }
+json.dump({"report": rep, "zones": zones, "kernels": out}, sys.stdout, indent=1)
+print()
