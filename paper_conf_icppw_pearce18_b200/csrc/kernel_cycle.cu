@@ -160,6 +160,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     issue(q0);
     issue(q0 + 1);
+    if (q0 + 2 <= k1 + 1) issue(q0 + 2);
   }
   __syncthreads();
 
@@ -190,23 +191,29 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   const int64_t gz_lo = -d.lo[2], gz_hi = d.N[2] - d.lo[2];  // plane q exists iff in [lo, hi)
   const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
 
-  double xpa, ypa, zpa;  // own node's x_p at plane p (corner 0 of the own zone)
+  // Software pipeline (3 barriers per plane, 4 when FUSED): iteration p runs
+  //   phase 1: E2 of zone plane p-2 and the zone/face stage of plane p,
+  //   phase 2: the node stage of node plane p,
+  //   phase 3: x_p of node plane p+2 and E1 of zone plane p-1.
+  double xpa, ypa, zpa, xpb, ypb, zpb;  // own node's x_p at planes p and p+1
   wait_plane(q0);
   form_xp(q0, xpa, ypa, zpa);
+  wait_plane(q0 + 1);
+  form_xp(q0 + 1, xpb, ypb, zpb);
+  double e2_P = 0.0, e2_e = 0.0, e2_im = 0.0, e2_part = 0.0;  // pending E2 of one zone plane
+  __syncthreads();
 
   for (int p = k0 - 1; p <= k1; ++p) {
-    // ---------------------------------------------------------------- X
-    if (t == 0 && p + 2 <= k1 + 1) issue(p + 2);  // slot of plane p-1, free since step p-1
+    // ---------------------------------------------------------------- phase 1: E2(p-2), Z(p)
+    if (p >= k0 + 2 && zone_owned_xy) {
+      const double Wk = 0.125 * e2_P * ((PSX[t + 1] + PSY[t + TXT]) + e2_part);
+      d.en[(int64_t)(p - 1) * zsxy + zoff] = e2_e - dt * Wk * e2_im;
+    }
     const bool exists = zone_xy_exists && p >= gz_lo && p < gz_hi;
-    wait_plane(p + 1);
-    double xpb, ypb, zpb;  // own node's x_p at plane p+1 (corner 4)
-    form_xp(p + 1, xpb, ypb, zpb);
     // zone plane p (TMA): m and e are 0 on zones outside the mesh (never written), P too
     double *MS = zraw(p), *ES = MS + ZRS, *PS = FUSED ? PSF : MS + 2 * ZRS;
     const double m = MS[tc], e = ES[tc];
     double P = FUSED ? 0.0 : PS[tc];
-    __syncthreads();
-    // ---------------------------------------------------------------- Z (+ G when not FUSED)
     const double *Ra = raw(p);
     const double *Xa = XP + (p & 1) * 3 * RS, *Xb = XP + ((p + 1) & 1) * 3 * RS;
     double im;
@@ -362,7 +369,13 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
       Msum_prev = Ms;
     }
     __syncthreads();
-    // ---------------------------------------------------------------- E
+    // ---------------------------------------------------------------- phase 3: X(p+2), E1(p-1)
+    if (t == 0 && p + 3 <= k1 + 1) issue(p + 3);  // slot of plane p, free after N(p)
+    double xpc = 0.0, ypc = 0.0, zpc = 0.0;
+    if (p + 2 <= k1 + 1) {
+      wait_plane(p + 2);
+      form_xp(p + 2, xpc, ypc, zpc);
+    }
     double psi_zhigh = 0.0, psx = 0.0, psy = 0.0;
     const double vsx = uhp + uh, vsy = vhp + vh, vsz = whp + wh;  // own two-plane u_half sum
     if (p >= k0) {
@@ -387,12 +400,13 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
                     cz0 * ((wh + a2_) + (b2 + c2_));
       }
     }
+    // E2 of zone plane p-1 runs in the next phase 1: W = P/8 (psi_xhi - psi_x + psi_yhi - psi_y
+    // + psi_zhi - psi_zlo) with the high-face psi read from the neighbours
+    e2_P = P_prev;
+    e2_e = e_prev;
+    e2_im = im_prev;
+    e2_part = ((psi_zhigh - psi_zlow) - psx) - psy;
     __syncthreads();
-    if (p >= k0 + 1 && zone_owned_xy) {
-      const double Wk = 0.125 * P_prev *
-                        (((PSX[t + 1] - psx) + (PSY[t + TXT] - psy)) + (psi_zhigh - psi_zlow));
-      d.en[(int64_t)p * zsxy + zoff] = e_prev - dt * Wk * im_prev;
-    }
     psi_zlow = psi_zhigh;
     P_prev = P;
     im_prev = im;
@@ -401,6 +415,11 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     bxp = bx0; byp = by0; bzp = bz0;
     uhp = uh; vhp = vh; whp = wh;
     xpa = xpb; ypa = ypb; zpa = zpb;
+    xpb = xpc; ypb = ypc; zpb = zpc;
+  }
+  if (k1 >= k0 + 1 && zone_owned_xy) {  // the last pending E2 (zone plane k1-1)
+    const double Wk = 0.125 * e2_P * ((PSX[t + 1] + PSY[t + TXT]) + e2_part);
+    d.en[(int64_t)k1 * zsxy + zoff] = e2_e - dt * Wk * e2_im;
   }
   if (FUSED) block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);
 }
