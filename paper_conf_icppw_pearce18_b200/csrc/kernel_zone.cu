@@ -21,6 +21,9 @@ namespace hydro {
 
 namespace {
 
+#ifndef HYDRO_ZONE_MINB
+#define HYDRO_ZONE_MINB 2
+#endif
 constexpr int ZBX = 32, ZBY = 8;                       // zones per block (x, y)
 constexpr int ZNX = ZONE_BOX_X, ZNY = ZBY + 1;         // TMA node box (x padded to 16 B)
 constexpr int ZNN = ZNX * ZNY;
@@ -33,7 +36,7 @@ constexpr int ZTOTAL = ZOFF_BAR + 4;
 constexpr size_t ZBYTES = ZTOTAL * sizeof(double);
 static_assert(ZNX >= ZBX + 2, "zone-kernel TMA box too narrow (33 nodes + 1 alignment shift)");
 
-__global__ void __launch_bounds__(ZBX *ZBY, 2)
+__global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
     k_zone_stage(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st,
                  int KZ, int zlox, int zloy, int zloz, int zhix, int zhiy, int zhiz) {
   const int3 zlo = make_int3(zlox, zloy, zloz), zhi = make_int3(zhix, zhiy, zhiz);
