@@ -359,9 +359,7 @@ def main():
         for _ in range(reps):
             hyd.set_state(pinned, pinned["e"], inf0["t"], inf0["dt"])
             hyd.step(args.e2e_cycles)
-            got = hyd.fields(names)
-            for k in names:
-                out[k][...] = got[k]
+            hyd.fields(names, out=out)
         el = time.perf_counter() - t0
         h2d = sum(v.nbytes for v in pinned.values())
         d2h = sum(v.nbytes for v in out.values())

@@ -60,7 +60,11 @@ void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s);
 
 // Intra-GPU ghost exchange of the next-parity state over a table of slab copies.
 void launch_halo_copy(const DomView *views_dev, const HaloCopy *pairs_dev, int npairs,
-                      cudaStream_t s);
+                      int blocks_per_pair, cudaStream_t s);
+
+// Strided 3-D box copy (src/dst pre-offset to the box origin; pitches in elements).
+void launch_copy3d(const double *src, int64_t ssx, int64_t ssxy, double *dst, int64_t dsx,
+                   int64_t dsxy, int ex, int ey, int ez, cudaStream_t s);
 
 // get_fields: derived zone fields (rho, p, q, c, vol) at (x, u) with no predictor into d.aux.
 void launch_derive(const DomView &d, const Phys &ph, cudaStream_t s);

@@ -303,6 +303,16 @@ __global__ void k_derive(DomView d, Phys ph) {
   d.aux[4 * d.nzone + id] = V;
 }
 
+// Strided 3-D box copy between device arrays (host transfers go through a contiguous staging
+// buffer: one full-bandwidth DMA plus this kernel, instead of a row-by-row 3-D memcpy).
+__global__ void k_copy3d(const double *__restrict__ src, int64_t ssx, int64_t ssxy,
+                         double *__restrict__ dst, int64_t dsx, int64_t dsxy, int ex) {
+  const int j = blockIdx.y, k = blockIdx.z;
+  const double *s = src + k * ssxy + j * ssx;
+  double *d = dst + k * dsxy + j * dsx;
+  for (int i = threadIdx.x; i < ex; i += blockDim.x) d[i] = s[i];
+}
+
 dim3 grid_for(int nx, int ny, int nz) {
   return dim3((nx + BX - 1) / BX, (ny + BY - 1) / BY, nz);
 }
@@ -338,10 +348,16 @@ void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s) {
   k_finalize<<<1, 1, 0, s>>>(st, ph);
 }
 void launch_halo_copy(const DomView *views_dev, const HaloCopy *pairs_dev, int npairs,
-                      cudaStream_t s) {
+                      int blocks_per_pair, cudaStream_t s) {
   if (npairs <= 0) return;
-  k_halo_copy<<<dim3(16, npairs), 256, 0, s>>>(views_dev, pairs_dev);
+  k_halo_copy<<<dim3(blocks_per_pair, npairs), 256, 0, s>>>(views_dev, pairs_dev);
 }
+void launch_copy3d(const double *src, int64_t ssx, int64_t ssxy, double *dst, int64_t dsx,
+                   int64_t dsxy, int ex, int ey, int ez, cudaStream_t s) {
+  if (ex <= 0 || ey <= 0 || ez <= 0) return;
+  k_copy3d<<<dim3(1, ey, ez), 128, 0, s>>>(src, ssx, ssxy, dst, dsx, dsxy, ex);
+}
+
 void launch_derive(const DomView &d, const Phys &ph, cudaStream_t s) {
   k_derive<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph);
 }

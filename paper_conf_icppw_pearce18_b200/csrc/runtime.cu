@@ -48,6 +48,7 @@ struct hydro_ctx {
   DomView *views_dev[2] = {nullptr, nullptr};
   HaloCopy *local_pairs_dev = nullptr;
   int n_local_pairs = 0;
+  int halo_blocks = 1;  // blocks per intra-GPU halo slab (sized by the largest slab)
   cudaGraphExec_t graph[2] = {nullptr, nullptr};
   int parity = 0;
   bool split = false;
@@ -55,6 +56,8 @@ struct hydro_ctx {
   bool use_graph = true;
   int failed = 0;
   Comm *comm = nullptr;
+  double *stage = nullptr;  // contiguous device staging for host transfers (lazy)
+  size_t stage_cap = 0;
   std::string err;
 };
 
@@ -166,6 +169,29 @@ int copy_box(hydro_ctx *h, bool to_device, double *host, const int64_t gdims[3],
              const int64_t glo[3], const int64_t ext[3], double *dev, int64_t dsx, int64_t dsy,
              const int64_t dlo_local[3], cudaStream_t s) {
   if (ext[0] <= 0 || ext[1] <= 0 || ext[2] <= 0) return HYDRO_OK;
+  double *dbox = dev + (dlo_local[2] * dsy + dlo_local[1]) * dsx + dlo_local[0];
+  if (ext[0] == gdims[0] && ext[1] == gdims[1]) {
+    // the host box is contiguous (whole planes): one full-bandwidth DMA through a device staging
+    // buffer and a strided copy kernel on the device
+    const size_t n = (size_t)ext[0] * ext[1] * ext[2];
+    if (n > h->stage_cap) {
+      if (h->stage) CK(cudaFreeAsync(h->stage, s));
+      CK(cudaMallocAsync(&h->stage, n * sizeof(double), s));
+      h->stage_cap = n;
+    }
+    double *hbox = host + (glo[2] * gdims[1] + glo[1]) * gdims[0] + glo[0];
+    if (to_device) {
+      CK(cudaMemcpyAsync(h->stage, hbox, n * sizeof(double), cudaMemcpyHostToDevice, s));
+      launch_copy3d(h->stage, ext[0], ext[0] * ext[1], dbox, dsx, dsx * dsy, (int)ext[0],
+                    (int)ext[1], (int)ext[2], s);
+    } else {
+      launch_copy3d(dbox, dsx, dsx * dsy, h->stage, ext[0], ext[0] * ext[1], (int)ext[0],
+                    (int)ext[1], (int)ext[2], s);
+      CK(cudaMemcpyAsync(hbox, h->stage, n * sizeof(double), cudaMemcpyDeviceToHost, s));
+    }
+    CK(cudaGetLastError());
+    return HYDRO_OK;
+  }
   cudaMemcpy3DParms p;
   std::memset(&p, 0, sizeof(p));
   cudaPitchedPtr hp = make_cudaPitchedPtr(host, gdims[0] * sizeof(double), gdims[0], gdims[1]);
@@ -254,7 +280,7 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
     }
     for (LocalDom &D : h->doms) launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, s);
   }
-  launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
+  launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, h->halo_blocks, s);
   if (h->comm) {
     int rc = comm_halo(h->comm, par, s);
     if (rc) return set_err(h, rc, "halo exchange failed");
@@ -458,6 +484,13 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
            }
          }
          h->n_local_pairs = (int)lp.size();
+         int64_t biggest = 0;
+         for (const HaloCopy &c : lp) {
+           int64_t nn = 1;
+           for (int a = 0; a < 3; ++a) nn *= c.nhi[a] - c.nlo[a];
+           biggest = std::max(biggest, nn);
+         }
+         h->halo_blocks = (int)std::max<int64_t>(1, std::min<int64_t>(1024, biggest / 1024));
          if (!lp.empty()) {
            CK(cudaMalloc(&h->local_pairs_dev, sizeof(HaloCopy) * lp.size()));
            CK(cudaMemcpyAsync(h->local_pairs_dev, lp.data(), sizeof(HaloCopy) * lp.size(),
@@ -672,7 +705,7 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
       for (LocalDom &D : h->doms) launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, s);
     }
     CK(cudaEventRecord(ev[1], s));
-    launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
+    launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, h->halo_blocks, s);
     if (h->comm && comm_halo(h->comm, par, s)) return HYDRO_ENCCL;
     CK(cudaEventRecord(ev[2], s));
     launch_finalize(h->st, h->ph, s);
@@ -719,6 +752,7 @@ int hydro_destroy(hydro_ctx *h) {
   for (LocalDom &D : h->doms)
     if (D.mem) cudaFree(D.mem);
   if (h->local_pairs_dev) cudaFree(h->local_pairs_dev);
+  if (h->stage) cudaFree(h->stage);
   if (h->st) cudaFree(h->st);
   if (h->stream) cudaStreamDestroy(h->stream);
   delete h;

@@ -310,21 +310,29 @@ class Hydro:
         self._L.hydro_get_info(self._h, C.byref(info))
         return _info(info)
 
-    def _arrays(self, names, node_shape, zone_shape, alloc=np.zeros):
+    def _arrays(self, names, node_shape, zone_shape, alloc=np.zeros, given=None):
         out = {}
         ptrs = (C.POINTER(C.c_double) * 13)()
         mask = 0
         for nm in names:
             f = ALL_FIELDS.index(nm)
-            arr = alloc(node_shape if f < 6 else zone_shape, dtype=np.float64)
+            shape = node_shape if f < 6 else zone_shape
+            if given is not None and nm in given:
+                arr = given[nm]
+                if arr.shape != shape or arr.dtype != np.float64 or not arr.flags.c_contiguous:
+                    raise ValueError(f"out[{nm!r}] must be a C-contiguous float64 array {shape}")
+            else:
+                arr = alloc(shape, dtype=np.float64)
             out[nm] = arr
             ptrs[f] = arr.ctypes.data_as(C.POINTER(C.c_double))
             mask |= 1 << f
         return out, ptrs, mask
 
-    def fields(self, names: Sequence[str] = ALL_FIELDS) -> Dict[str, np.ndarray]:
+    def fields(self, names: Sequence[str] = ALL_FIELDS,
+               out: Optional[Dict[str, np.ndarray]] = None) -> Dict[str, np.ndarray]:
+        """Global fields; ``out`` may supply caller-owned (e.g. pinned) arrays to fill."""
         nx, ny, nz = (int(v) for v in self.cfg.n)
-        out, ptrs, mask = self._arrays(names, (nz + 1, ny + 1, nx + 1), (nz, ny, nx))
+        out, ptrs, mask = self._arrays(names, (nz + 1, ny + 1, nx + 1), (nz, ny, nx), given=out)
         rc = self._L.hydro_get_fields(self._h, mask, ptrs)
         if rc != 0:
             raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
