@@ -18,6 +18,7 @@
 //      e' = e - dt W / m (S8), written to HBM.
 // No tensor cores: nothing here is a dense contraction (BASELINE.json north_star).
 #include <algorithm>
+#include <climits>
 #include <cmath>
 
 #include "fastmath.cuh"
@@ -172,23 +173,33 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   double psi_zlow = 0.0;
   double dt2min = INFINITY;
 
-  const int64_t gxz = d.lo[0] + li, gyz = d.lo[1] + lj;
-  const bool zone_xy_exists = active && li <= n0 && lj <= n1 && gxz >= 0 && gxz < d.N[0] &&
-                              gyz >= 0 && gyz < d.N[1];
-  const bool node_xy = active && tx >= 1 && ty >= 1 && li <= n0 && lj <= n1;
-  const bool node_write_xy = node_xy && (li < i0 + TX || li == n0) && (lj < j0 + TY || lj == n1);
-  const bool zone_owned_xy = active && tx >= 1 && ty >= 1 && tx <= TX && ty <= TY && li < n0 &&
-                             lj < n1;
-  const bool ex_x = active && tx >= 1 && tx <= TX + 1 && ty >= 1 && ty <= TY;
-  const bool ex_y = active && tx >= 1 && tx <= TX && ty >= 1 && ty <= TY + 1;
-  const bool ex_z = active && tx >= 1 && tx <= TX && ty >= 1 && ty <= TY;
+  // Per-thread constants, kept in few registers (32-bit indices: a domain's storage is below
+  // 2^31 elements, checked at create) so the compiler does not rematerialise them per plane.
+  const int gxz = (int)d.lo[0] + li, gyz = (int)d.lo[1] + lj;
   const uint32_t rm = ph.reflect_mask;
-  const bool wall_x = (gxz == 0 && (rm & 1u)) || (gxz == d.N[0] && (rm & 2u));
-  const bool wall_y = (gyz == 0 && (rm & 4u)) || (gyz == d.N[1] && (rm & 8u));
-  const int64_t zsxy = d.zsxy, nsxy = d.nsxy;
-  const int64_t zoff = (int64_t)(lj + 1) * d.zsx + (li + 1);  // + (q+1)*zsxy
-  const int64_t nrow = (int64_t)(lj + 1) * d.nsx + (li + 1);
-  const int64_t gz_lo = -d.lo[2], gz_hi = d.N[2] - d.lo[2];  // plane q exists iff in [lo, hi)
+  enum : uint32_t { F_ZEX = 1, F_NODE = 2, F_NWR = 4, F_OWN = 8, F_EXX = 16, F_EXY = 32,
+                    F_EXZ = 64, F_WX = 128, F_WY = 256 };
+  uint32_t fl = 0;
+  {
+    const bool in_t = active && tx >= 1 && ty >= 1;
+    if (active && li <= n0 && lj <= n1 && gxz >= 0 && gxz < d.N[0] && gyz >= 0 && gyz < d.N[1])
+      fl |= F_ZEX;
+    if (in_t && li <= n0 && lj <= n1) {
+      fl |= F_NODE;
+      if ((li < i0 + TX || li == n0) && (lj < j0 + TY || lj == n1)) fl |= F_NWR;
+    }
+    if (in_t && tx <= TX && ty <= TY && li < n0 && lj < n1) fl |= F_OWN;
+    if (in_t && tx <= TX + 1 && ty <= TY) fl |= F_EXX;
+    if (in_t && tx <= TX && ty <= TY + 1) fl |= F_EXY;
+    if (in_t && tx <= TX && ty <= TY) fl |= F_EXZ;
+    if ((gxz == 0 && (rm & 1u)) || (gxz == d.N[0] && (rm & 2u))) fl |= F_WX;
+    if ((gyz == 0 && (rm & 4u)) || (gyz == d.N[1] && (rm & 8u))) fl |= F_WY;
+  }
+  const int zsxy = (int)d.zsxy, nsxy = (int)d.nsxy;
+  const int zoff = (lj + 1) * (int)d.zsx + (li + 1);  // zone id = (q+1)*zsxy + zoff
+  const int nrow = (lj + 1) * (int)d.nsx + (li + 1);  // node id = (q+1)*nsxy + nrow
+  const int gz_lo = -(int)d.lo[2], gz_hi = d.N[2] - (int)d.lo[2];  // plane q exists iff in range
+  const int wz_lo = (rm & 16u) ? gz_lo : INT_MIN, wz_hi = (rm & 32u) ? gz_hi : INT_MIN;
   const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
 
   // Software pipeline (3 barriers per plane, 4 when FUSED): iteration p runs
@@ -205,11 +216,11 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
 
   for (int p = k0 - 1; p <= k1; ++p) {
     // ---------------------------------------------------------------- phase 1: E2(p-2), Z(p)
-    if (p >= k0 + 2 && zone_owned_xy) {
+    if (p >= k0 + 2 && (fl & F_OWN)) {
       const double Wk = 0.125 * e2_P * ((PSX[t + 1] + PSY[t + TXT]) + e2_part);
-      d.en[(int64_t)(p - 1) * zsxy + zoff] = e2_e - dt * Wk * e2_im;
+      d.en[(p - 1) * zsxy + zoff] = e2_e - dt * Wk * e2_im;
     }
-    const bool exists = zone_xy_exists && p >= gz_lo && p < gz_hi;
+    const bool exists = (fl & F_ZEX) && p >= gz_lo && p < gz_hi;
     // zone plane p (TMA): m and e are 0 on zones outside the mesh (never written), P too
     double *MS = zraw(p), *ES = MS + ZRS, *PS = FUSED ? PSF : MS + 2 * ZRS;
     const double m = MS[tc], e = ES[tc];
@@ -276,7 +287,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
         qr = s * (ph.q_quad * s + ph.q_lin * c);
       }
       P = exists ? pr + rho * qr : 0.0;
-      if (exists && p >= k0 && p < k1 && zone_owned_xy) {
+      if (exists && p >= k0 && p < k1 && (fl & F_OWN)) {
         const double V2 = V * V;
         const double n1c = cfl4 * V2, d1c = (c2 + 2.0 * qr) * a2;
         const double n2c = cv2 * V2, d2c = DV * DV;
@@ -286,7 +297,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
         const double dt2 = (ok1 || ok2) ? num * frcp(den) : INFINITY;
         dt2min = dt2 < dt2min ? dt2 : dt2min;
         if (!(V > 0.0) || !isfinite(P)) {
-          const int64_t gzi = ((d.lo[2] + p) * d.N[1] + gyz) * (int64_t)d.N[0] + gxz;
+          const int64_t gzi = ((d.lo[2] + p) * d.N[1] + gyz) * (int64_t)d.N[0] + gxz;  // global
           flag_error_zone(st, (V > 0.0) ? ERR_NONFINITE : ERR_TANGLED, gzi);
         }
       }
@@ -325,7 +336,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     __syncthreads();
     // ---------------------------------------------------------------- N
     double uh = 0.0, vh = 0.0, wh = 0.0;
-    if (node_xy) {
+    if (fl & F_NODE) {
       const int tn = tc - TXT;  // zone (tx, ty-1)
       double a0, a1, a2_, b0, b1, b2;
       ld3(GX, tn, a0, a1, a2_);      // g_x of zone (tx, ty-1)
@@ -343,10 +354,9 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
         const double Fy = Sy + Cy + ((a1 + b1) + (c1 + gzy));
         const double Fz = Sz + Cz + ((a2_ + b2) + (c2_ + gzz));
         const double rinv = 8.0 * frcp(Msum_prev + Ms);
-        const int64_t g2 = d.lo[2] + p;
-        const bool wall_z = (g2 == 0 && (rm & 16u)) || (g2 == d.N[2] && (rm & 32u));
-        const double axc = wall_x ? 0.0 : Fx * rinv;
-        const double ayc = wall_y ? 0.0 : Fy * rinv;
+        const bool wall_z = p == wz_lo || p == wz_hi;
+        const double axc = (fl & F_WX) ? 0.0 : Fx * rinv;
+        const double ayc = (fl & F_WY) ? 0.0 : Fy * rinv;
         const double azc = wall_z ? 0.0 : Fz * rinv;
         const double u = Ra[3 * RS + nidx], v = Ra[4 * RS + nidx], w = Ra[5 * RS + nidx];
         const double un = u + dt * axc, vn = v + dt * ayc, wn = w + dt * azc;
@@ -355,8 +365,8 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
         wh = (w + wn) * 0.5;
         st3(UH, tc, uh, vh, wh);
         st3(VS, tc, uhp + uh, vhp + vh, whp + wh);
-        if (node_write_xy && (p < k1 || p == n2)) {
-          const int64_t id = (int64_t)(p + 1) * nsxy + nrow;
+        if ((fl & F_NWR) && (p < k1 || p == n2)) {
+          const int id = (p + 1) * nsxy + nrow;
           d.xn[id] = Ra[nidx] + dt * uh;
           d.yn[id] = Ra[RS + nidx] + dt * vh;
           d.zn[id] = Ra[2 * RS + nidx] + dt * wh;
@@ -381,18 +391,18 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     if (p >= k0) {
       double a0, a1, a2_, b0, b1, b2, c0, c1, c2_;
       if (p >= k0 + 1) {
-        if (ex_x) {  // x-low face of zone plane p-1: nodes (tx, ty..ty+1), planes p-1, p
+        if (fl & F_EXX) {  // x-low face of zone plane p-1: nodes (tx, ty..ty+1), planes p-1, p
           ld3(VS, tc + TXT, a0, a1, a2_);
           psx = axp * (vsx + a0) + ayp * (vsy + a1) + azp * (vsz + a2_);
           PSX[t] = psx;
         }
-        if (ex_y) {  // y-low face of zone plane p-1: nodes (tx..tx+1, ty), planes p-1, p
+        if (fl & F_EXY) {  // y-low face of zone plane p-1: nodes (tx..tx+1, ty), planes p-1, p
           ld3(VS, tc + 1, a0, a1, a2_);
           psy = bxp * (vsx + a0) + byp * (vsy + a1) + bzp * (vsz + a2_);
           PSY[t] = psy;
         }
       }
-      if (ex_z) {  // z-face at node plane p: nodes (tx..tx+1, ty..ty+1)
+      if (fl & F_EXZ) {  // z-face at node plane p: nodes (tx..tx+1, ty..ty+1)
         ld3(UH, tc + 1, a0, a1, a2_);
         ld3(UH, tc + TXT, b0, b1, b2);
         ld3(UH, tc + TXT + 1, c0, c1, c2_);
@@ -417,9 +427,9 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     xpa = xpb; ypa = ypb; zpa = zpb;
     xpb = xpc; ypb = ypc; zpb = zpc;
   }
-  if (k1 >= k0 + 1 && zone_owned_xy) {  // the last pending E2 (zone plane k1-1)
+  if (k1 >= k0 + 1 && (fl & F_OWN)) {  // the last pending E2 (zone plane k1-1)
     const double Wk = 0.125 * e2_P * ((PSX[t + 1] + PSY[t + TXT]) + e2_part);
-    d.en[(int64_t)k1 * zsxy + zoff] = e2_e - dt * Wk * e2_im;
+    d.en[k1 * zsxy + zoff] = e2_e - dt * Wk * e2_im;
   }
   if (FUSED) block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);
 }

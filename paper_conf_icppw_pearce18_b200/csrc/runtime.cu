@@ -83,6 +83,8 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
   // row pitches padded to 4 doubles (32 B): TMA needs 16-byte strides
   const int64_t nsx = (n0 + 3 + 3) / 4 * 4, nsxy = nsx * (n1 + 3), nnode = nsxy * (n2 + 3);
   const int64_t zsx = (n0 + 2 + 3) / 4 * 4, zsxy = zsx * (n1 + 2), nzone = zsxy * (n2 + 2);
+  if (nnode >= (int64_t(1) << 31))  // the cycle kernels index a domain's storage with int32
+    return set_err(h, HYDRO_EINVAL, "domain too large: split it into more domains (< 2^31 nodes)");
   const size_t nb = align_up(nnode * sizeof(double), 256), zb = align_up(nzone * sizeof(double), 256);
   // 12 node arrays (2 parities x 6), e x2, m, P, aux x5, optional B x24
   size_t bytes = 12 * nb + 9 * zb + (split ? 24 * zb : 0);
