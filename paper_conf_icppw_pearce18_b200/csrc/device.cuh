@@ -57,9 +57,50 @@ struct DevState {
   unsigned int err;             // error bits raised during the current cycle
   unsigned int halted;          // != 0: run stopped with these error bits
   unsigned int done;            // t >= t_stop
-  unsigned int pad_;
+  unsigned int blocks_done;     // CTAs of the last cycle kernel that finished (folded finalize)
 };
 
 enum : unsigned int { ERR_TANGLED = 1u, ERR_NONFINITE = 2u };
+
+// S9: t' = t + dt, dt' = min(min(growth*dt, dt_max), min_z dt_z), t_stop clamp;
+// latch the cycle's error bits so later cycles become no-ops (the state stays the one after the
+// failing cycle, as in the oracle).  Run by one thread after every kernel of the cycle.
+__device__ __forceinline__ void finalize_cycle(DevState *st, const Phys &ph) {
+  if (st->halted | st->done) return;
+  const double dtmin = __longlong_as_double((long long)st->dtz_acc);
+  const double dt = st->dt;
+  const double tn = st->t + dt;
+  double dtn = fmin(fmin(ph.dt_growth * dt, ph.dt_max), dtmin);
+  const bool stop = ph.t_stop > 0.0 && tn >= ph.t_stop;
+  if (ph.t_stop > 0.0) dtn = fmin(dtn, ph.t_stop - tn);
+  st->t = tn;
+  st->dt = dtn;
+  st->dtz_last = dtmin;
+  st->cycle += 1;
+  st->dtz_acc = (unsigned long long)__double_as_longlong(INFINITY);
+  unsigned err = st->err;
+  if (!(isfinite(dtn) && dtn > 0.0) && !stop) err |= ERR_NONFINITE;
+  st->halted = err;
+  st->done = stop ? 1u : 0u;
+}
+
+// Folded finalize: the last CTA of a kernel to finish runs finalize_cycle (every other CTA has
+// read st->dt before finishing).  Call from all threads at the very end of the kernel; ticket is
+// one word of shared scratch.
+__device__ __forceinline__ void finalize_if_last_block(DevState *st, const Phys &ph,
+                                                       unsigned int *ticket) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    *ticket = atomicAdd(&st->blocks_done, 1u);
+  }
+  __syncthreads();
+  const unsigned total = gridDim.x * gridDim.y * gridDim.z;
+  if (threadIdx.x == 0 && *ticket == total - 1) {
+    __threadfence();
+    finalize_cycle(st, ph);
+    st->blocks_done = 0;
+  }
+}
 
 }  // namespace hydro

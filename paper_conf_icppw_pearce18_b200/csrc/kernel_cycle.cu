@@ -64,7 +64,8 @@ struct CTile {
 
 template <int TX, int TY, bool FUSED>
 __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
-    k_cycle(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st, int KZ) {
+    k_cycle(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st, int KZ,
+            int fold_finalize) {
   using T = CTile<TX, TY>;
   // dynamic shared memory only (no static __shared__), so the window is 1024-byte aligned
   extern __shared__ __align__(1024) double sm[];
@@ -432,6 +433,8 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     d.en[k1 * zsxy + zoff] = e2_e - dt * Wk * e2_im;
   }
   if (FUSED) block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);
+  if (fold_finalize)  // single-domain, single-rank cycle: S9 here instead of a separate launch
+    finalize_if_last_block(st, ph, reinterpret_cast<unsigned int *>(sm + T::OFF_RED));
 }
 
 constexpr int CTX = 32, CTY = 12;
@@ -452,7 +455,8 @@ int choose_kz(int tiles, int n2, int sms) {
 }
 
 template <bool FUSED>
-void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st, cudaStream_t s) {
+void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st, int fold,
+            cudaStream_t s) {
   using T = CTile<CTX, CTY>;
   static int sms = 0;
   if (!sms) {
@@ -465,7 +469,7 @@ void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st
   const int tx = (d.n[0] + CTX - 1) / CTX, ty = (d.n[1] + CTY - 1) / CTY;
   const int KZ = choose_kz(tx * ty, d.n[2], sms);
   dim3 grid(tx, ty, (d.n[2] + KZ - 1) / KZ);
-  k_cycle<CTX, CTY, FUSED><<<grid, T::NTHR, T::BYTES, s>>>(maps, d, ph, st, KZ);
+  k_cycle<CTX, CTY, FUSED><<<grid, T::NTHR, T::BYTES, s>>>(maps, d, ph, st, KZ, fold);
 }
 
 }  // namespace
@@ -477,13 +481,13 @@ int cycle_zone_box_x() { return CTile<CTX, CTY>::ZBX; }
 int cycle_zone_box_y() { return CTile<CTX, CTY>::ZBY; }
 
 void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                        cudaStream_t s) {
-  launch<true>(d, maps, ph, st, s);
+                        int fold_finalize, cudaStream_t s) {
+  launch<true>(d, maps, ph, st, fold_finalize, s);
 }
 
 void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                        cudaStream_t s) {
-  launch<false>(d, maps, ph, st, s);
+                        int fold_finalize, cudaStream_t s) {
+  launch<false>(d, maps, ph, st, fold_finalize, s);
 }
 
 }  // namespace hydro

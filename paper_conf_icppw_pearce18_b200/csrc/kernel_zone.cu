@@ -111,6 +111,7 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
     e_nx = d.e[(int64_t)(zk0 + 1) * d.zsxy + zrow];
   }
 
+  double zlx = 0.0, zly = 0.0, zlz = 0.0;  // z-high face of the zone below (carried)
   for (int p = zk0; p < zk1; ++p) {
     const double m = m_nx, e = e_nx;
     const bool exists = exists_xy && p >= gz_lo && p < gz_hi;
@@ -142,16 +143,27 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
 #pragma unroll
     for (int b = 0; b < 2; ++b)
       HYDRO_FACE(X, Y, Z, 5 + 2 * b, 2 * b, 1 + 2 * b, 2 * b + 4, fx[2 + b], fy[2 + b], fz[2 + b]);
+    // z-low face = the z-high face this thread formed for the zone below (same nodes, same bits)
+    if (p == zk0) HYDRO_FACE(X, Y, Z, 3, 0, 2, 1, zlx, zly, zlz);
+    fx[4] = zlx; fy[4] = zly; fz[4] = zlz;
+    HYDRO_FACE(X, Y, Z, 7, 4, 6, 5, fx[5], fy[5], fz[5]);
+    zlx = fx[5]; zly = fy[5]; zlz = fz[5];
+    // corner vectors S_l = s(a)AX_a + (s(b)AY_b + s(c)AZ_c): the (b, c) pair sums once
+    double qx[4], qy[4], qz[4];
 #pragma unroll
-    for (int c = 0; c < 2; ++c)
-      HYDRO_FACE(X, Y, Z, 3 + 4 * c, 4 * c, 2 + 4 * c, 1 + 4 * c, fx[4 + c], fy[4 + c], fz[4 + c]);
+    for (int bc = 0; bc < 4; ++bc) {
+      const int b = bc & 1, c = bc >> 1;
+      qx[bc] = (b ? fx[3] : -fx[2]) + (c ? fx[5] : -fx[4]);
+      qy[bc] = (b ? fy[3] : -fy[2]) + (c ? fy[5] : -fy[4]);
+      qz[bc] = (b ? fz[3] : -fz[2]) + (c ? fz[5] : -fz[4]);
+    }
     double V8 = 0.0, DV8 = 0.0;
 #pragma unroll
     for (int l = 0; l < 8; ++l) {
-      const int a = l & 1, b = (l >> 1) & 1, c = (l >> 2) & 1;
-      const double sx = (a ? fx[1] : -fx[0]) + (b ? fx[3] : -fx[2]) + (c ? fx[5] : -fx[4]);
-      const double sy = (a ? fy[1] : -fy[0]) + (b ? fy[3] : -fy[2]) + (c ? fy[5] : -fy[4]);
-      const double sz = (a ? fz[1] : -fz[0]) + (b ? fz[3] : -fz[2]) + (c ? fz[5] : -fz[4]);
+      const int a = l & 1, b = (l >> 1) & 1, c = (l >> 2) & 1, bc = l >> 1;
+      const double sx = (a ? fx[1] : -fx[0]) + qx[bc];
+      const double sy = (a ? fy[1] : -fy[0]) + qy[bc];
+      const double sz = (a ? fz[1] : -fz[0]) + qz[bc];
       if (l > 0) V8 += (X[l] - X[0]) * sx + (Y[l] - Y[0]) * sy + (Z[l] - Z[0]) * sz;
       const double *Us = c ? Ub : Ua;
       const int n = nidx + b * ZNX + a;

@@ -40,8 +40,10 @@ struct alignas(64) NodeMaps {
 };
 
 // Fused single-kernel cycle (default path).
+// fold_finalize != 0: the kernel's last CTA also performs S9 (k_finalize is then not launched;
+// only valid when this is the cycle's last kernel: one domain, one rank).
 void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                        cudaStream_t s);
+                        int fold_finalize, cudaStream_t s);
 size_t fused_smem_bytes();
 int fused_box_y();
 
@@ -49,7 +51,7 @@ int fused_box_y();
 void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                        cudaStream_t s);
 void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                        cudaStream_t s);
+                        int fold_finalize, cudaStream_t s);
 int zone_box_y();
 int node_box_y();
 int cycle_zone_box_x();  // zone-field TMA box of the cycle kernels

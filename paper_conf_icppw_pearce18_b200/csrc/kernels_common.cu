@@ -122,27 +122,8 @@ __global__ void k_finalize_init(DevState *st, double dt_first, double dt_init, d
   st->done = (t_stop > 0.0 && t0 >= t_stop) ? 1u : 0u;
 }
 
-// S9: t' = t + dt, dt' = min(min(growth*dt, dt_max), min_z dt_z), t_stop clamp;
-// latch the cycle's error bits so later cycles become no-ops (the state stays the one after the
-// failing cycle, as in the oracle).
-__global__ void k_finalize(DevState *st, Phys ph) {
-  if (st->halted | st->done) return;
-  const double dtmin = __longlong_as_double((long long)st->dtz_acc);
-  const double dt = st->dt;
-  const double tn = st->t + dt;
-  double dtn = fmin(fmin(ph.dt_growth * dt, ph.dt_max), dtmin);
-  const bool stop = ph.t_stop > 0.0 && tn >= ph.t_stop;
-  if (ph.t_stop > 0.0) dtn = fmin(dtn, ph.t_stop - tn);
-  st->t = tn;
-  st->dt = dtn;
-  st->dtz_last = dtmin;
-  st->cycle += 1;
-  st->dtz_acc = (unsigned long long)__double_as_longlong(INFINITY);
-  unsigned err = st->err;
-  if (!(isfinite(dtn) && dtn > 0.0) && !stop) err |= ERR_NONFINITE;
-  st->halted = err;
-  st->done = stop ? 1u : 0u;
-}
+// S9 as its own kernel (multi-domain / multi-rank cycles; see finalize_cycle).
+__global__ void k_finalize(DevState *st, Phys ph) { finalize_cycle(st, ph); }
 
 // ------------------------------------------------------------------ split pipeline
 // K1: S1-S6 for every existing local zone (owned and ghost): P and the 24 corner-vector

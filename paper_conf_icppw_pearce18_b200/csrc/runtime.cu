@@ -254,6 +254,18 @@ int upload_state(hydro_ctx *h, int par, const double *const *nodes6, const doubl
   return HYDRO_OK;
 }
 
+// S9 can run inside the cycle's last kernel when that kernel is the only one of the cycle (one
+// domain, one rank, not the plain split path).  Measured on B200 at 128^3 it is slower (the
+// per-CTA __threadfence before the ticket delays every CTA's exit: node stage 106 -> 110 us,
+// while a separate k_finalize costs ~2.6 us), so it is off unless built with -DHYDRO_FOLD.
+int fold_finalize(const hydro_ctx *h) {
+#ifndef HYDRO_FOLD
+  (void)h;
+  return 0;
+#endif
+  return (!h->split && h->doms.size() == 1 && !h->comm && h->n_local_pairs == 0) ? 1 : 0;
+}
+
 // Enqueue one cycle on stream s reading parity `par`.
 int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
   for (LocalDom &D : h->doms) {
@@ -269,7 +281,7 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
     for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
     for (LocalDom &D : h->doms) launch_energy_split(D.view[par], h->ph, h->st, s);
   } else if (h->one_kernel) {
-    for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, s);
+    for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
     if (h->comm) {
       int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
@@ -280,14 +292,14 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
       int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
     }
-    for (LocalDom &D : h->doms) launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, s);
+    for (LocalDom &D : h->doms) launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
   }
   launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, h->halo_blocks, s);
   if (h->comm) {
     int rc = comm_halo(h->comm, par, s);
     if (rc) return set_err(h, rc, "halo exchange failed");
   }
-  launch_finalize(h->st, h->ph, s);
+  if (!fold_finalize(h)) launch_finalize(h->st, h->ph, s);
   CK(cudaGetLastError());
   return HYDRO_OK;
 }
@@ -675,7 +687,7 @@ int hydro_kernels_per_cycle(const hydro_ctx *h) {
   const int nd = (int)h->doms.size();
   int k = (h->split ? 3 : (h->one_kernel ? 1 : 2)) * nd;  // cycle kernels
   if (h->n_local_pairs > 0) k += 1;  // intra-GPU halo copy
-  k += 1;                            // finalize
+  if (!fold_finalize(h)) k += 1;     // finalize
   if (h->comm) k += comm_kernels_per_cycle(h->comm);
   return k;
 }
@@ -698,19 +710,19 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
       for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
       for (LocalDom &D : h->doms) launch_energy_split(D.view[par], h->ph, h->st, s);
     } else if (h->one_kernel) {
-      for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, s);
+      for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
       if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
     } else {
       for (LocalDom &D : h->doms) launch_zone_stage(D.view[par], D.zmaps[par], h->ph, h->st, s);
       if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
       CK(cudaEventRecord(ev[4], s));
-      for (LocalDom &D : h->doms) launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, s);
+      for (LocalDom &D : h->doms) launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
     }
     CK(cudaEventRecord(ev[1], s));
     launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, h->halo_blocks, s);
     if (h->comm && comm_halo(h->comm, par, s)) return HYDRO_ENCCL;
     CK(cudaEventRecord(ev[2], s));
-    launch_finalize(h->st, h->ph, s);
+    if (!fold_finalize(h)) launch_finalize(h->st, h->ph, s);
     CK(cudaEventRecord(ev[3], s));
     CK(cudaEventSynchronize(ev[3]));
     float a, b, cc, d;
