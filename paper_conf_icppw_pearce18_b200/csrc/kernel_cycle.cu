@@ -20,6 +20,7 @@
 #include <algorithm>
 #include <climits>
 #include <cmath>
+#include <cstdlib>
 
 #include "fastmath.cuh"
 #include "kernels.h"
@@ -467,7 +468,9 @@ void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st
                          (int)T::BYTES);
   }
   const int tx = (d.n[0] + CTX - 1) / CTX, ty = (d.n[1] + CTY - 1) / CTY;
-  const int KZ = choose_kz(tx * ty, d.n[2], sms);
+  static const int kz_env = getenv(FUSED ? "HYDRO_KZ_FUSED" : "HYDRO_KZ_NODE")
+                                ? atoi(getenv(FUSED ? "HYDRO_KZ_FUSED" : "HYDRO_KZ_NODE")) : 0;
+  const int KZ = kz_env > 0 ? std::min(kz_env, d.n[2]) : choose_kz(tx * ty, d.n[2], sms);
   dim3 grid(tx, ty, (d.n[2] + KZ - 1) / KZ);
   k_cycle<CTX, CTY, FUSED><<<grid, T::NTHR, T::BYTES, s>>>(maps, d, ph, st, KZ, fold);
 }

@@ -11,6 +11,7 @@
 // ring per tile.
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 
 #include "fastmath.cuh"
 #include "kernels.h"
@@ -249,7 +250,8 @@ void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, D
   }
   const int nz_x = hi[0] - lo[0], nz_y = hi[1] - lo[1], nz_z = hi[2] - lo[2];
   const int tx = (nz_x + ZBX - 1) / ZBX, ty = (nz_y + ZBY - 1) / ZBY;
-  const int KZ = choose_kz_zone(tx * ty, nz_z, slots);
+  static const int kz_env = getenv("HYDRO_KZ_ZONE") ? atoi(getenv("HYDRO_KZ_ZONE")) : 0;
+  const int KZ = kz_env > 0 ? std::min(kz_env, nz_z) : choose_kz_zone(tx * ty, nz_z, slots);
   dim3 grid(tx, ty, (nz_z + KZ - 1) / KZ);
   k_zone_stage<<<grid, ZBX * ZBY, ZBYTES, s>>>(maps, d, ph, st, KZ, lo[0], lo[1], lo[2], hi[0],
                                                hi[1], hi[2]);
