@@ -435,6 +435,7 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
   h->device = cfg->device;
   *out = nullptr;
   auto fail = [&](int code) {
+    if (!h->err.empty()) g_err = h->err;  // hydro_last_error(NULL) after a failed create
     hydro_destroy(h);
     return code;
   };
