@@ -8,6 +8,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <limits>
 #include <string>
@@ -266,6 +267,10 @@ int fold_finalize(const hydro_ctx *h) {
   return (!h->split && h->doms.size() == 1 && !h->comm && h->n_local_pairs == 0) ? 1 : 0;
 }
 
+void launch_node_stage(hydro_ctx *h, LocalDom &D, int par, cudaStream_t s) {
+  launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
+}
+
 // Enqueue one cycle on stream s reading parity `par`.
 int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
   for (LocalDom &D : h->doms) {
@@ -292,7 +297,7 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
       int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
     }
-    for (LocalDom &D : h->doms) launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
+    for (LocalDom &D : h->doms) launch_node_stage(h, D, par, s);
   }
   launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, h->halo_blocks, s);
   if (h->comm) {
@@ -717,7 +722,7 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
       for (LocalDom &D : h->doms) launch_zone_stage(D.view[par], D.zmaps[par], h->ph, h->st, s);
       if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
       CK(cudaEventRecord(ev[4], s));
-      for (LocalDom &D : h->doms) launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
+      for (LocalDom &D : h->doms) launch_node_stage(h, D, par, s);
     }
     CK(cudaEventRecord(ev[1], s));
     launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, h->halo_blocks, s);
