@@ -237,6 +237,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--path", default="two", choices=["two", "one", "split"],
                     help="two: zone + node/energy kernels; one: one fused kernel; split: plain")
+    ap.add_argument("--transport", default="peer", choices=["peer", "nccl"],
+                    help="N>1 halo/dt transport: CUDA IPC peer stores (tested with 2 ranks on one "
+                         "GPU) or NCCL send/recv + allreduce")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-cycles", type=int, default=100)
     args = ap.parse_args()
@@ -257,7 +260,8 @@ def main():
     from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig
 
     kw, scaling, desc = workload(args.config, ngpu)
-    cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, path=args.path, **kw)
+    cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, path=args.path,
+                      transport=args.transport, **kw)
     hyd = Hydro(cfg)
     n = kw["n"]
     zones = n[0] * n[1] * n[2]
@@ -380,7 +384,8 @@ def main():
                        "zones": zones, "path": args.path,
                        "l2": "state > 126 MB L2 (inputs larger than L2; no flush)"
                        if zones * 120 > 126e6 else "state fits L2",
-                       "parallelism": f"dp{ngpu} (spatial domains)"},
+                       "parallelism": f"dp{ngpu} (spatial domains)",
+                       "transport": args.transport if ngpu > 1 else None},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clk.summary(),
             "gpu_launches": launches, "kernel_ms": kt,
         }

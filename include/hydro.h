@@ -68,6 +68,9 @@ enum {
 #define HYDRO_FLAG_SPLIT (1ull << 1)    /* plain 3-kernel pipeline (one thread per element) */
 #define HYDRO_FLAG_ONE_KERNEL (1ull << 2) /* one fused kernel per cycle (zone ring recomputed)
                                              instead of the default zone + node/energy pair */
+#define HYDRO_FLAG_PEER (1ull << 3)       /* nranks > 1: exchange halos and reduce dt through peer
+                                             memory (CUDA IPC; ranks may share a GPU) instead of
+                                             NCCL; needs hydro_peer_export/import after create */
 
 typedef struct {
   int32_t abi_version;          /* must be HYDRO_ABI_VERSION */
@@ -146,6 +149,15 @@ int hydro_get_box(hydro_ctx *h, const int64_t lo[3], const int64_t hi[3], uint32
    (host -> device copies through the public API).  Clears a failed state.  Collective. */
 int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, double t,
                     double dt);
+
+/* Peer transport (HYDRO_FLAG_PEER) bootstrap, collective: after hydro_create every rank calls
+   hydro_peer_export (buf NULL: *len = bytes needed), the caller all-gathers the records (padded to
+   a common len_per_rank, rank order), and every rank calls hydro_peer_import with all of them;
+   import maps the neighbours' domain allocations and mailboxes, reduces dt^0 over the ranks and
+   captures the cycle graphs.  hydro_step returns HYDRO_ESTATE before import.
+   Errors: HYDRO_EINVAL (bad records), HYDRO_ECUDA (IPC failures). */
+int hydro_peer_export(hydro_ctx *h, void *buf, size_t *len);
+int hydro_peer_import(hydro_ctx *h, const void *all, size_t len_per_rank);
 
 /* Current info without stepping. */
 int hydro_get_info(hydro_ctx *h, hydro_info *info);

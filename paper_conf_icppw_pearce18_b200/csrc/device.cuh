@@ -58,6 +58,7 @@ struct DevState {
   unsigned int halted;          // != 0: run stopped with these error bits
   unsigned int done;            // t >= t_stop
   unsigned int blocks_done;     // CTAs of the last cycle kernel that finished (folded finalize)
+  unsigned long long xchg;      // peer-transport exchange epoch (peer.cu)
 };
 
 enum : unsigned int { ERR_TANGLED = 1u, ERR_NONFINITE = 2u };

@@ -18,6 +18,7 @@
 #include "comm.h"
 #include "kernels.h"
 #include "layout.h"
+#include "peer.h"
 
 using namespace hydro;
 
@@ -57,6 +58,7 @@ struct hydro_ctx {
   bool use_graph = true;
   int failed = 0;
   Comm *comm = nullptr;
+  Peer *peer = nullptr;      // HYDRO_FLAG_PEER transport (nranks > 1)
   double *stage = nullptr;  // contiguous device staging for host transfers (lazy)
   size_t stage_cap = 0;
   std::string err;
@@ -79,20 +81,27 @@ int set_err(hydro_ctx *h, int code, const std::string &msg) {
 
 size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 
-int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
-  const int64_t n0 = D.box.n[0], n1 = D.box.n[1], n2 = D.box.n[2];
+}  // namespace
+
+namespace hydro {
+
+// Storage of one domain inside its single allocation (also used to reconstruct the arrays of a
+// remote domain from its IPC-mapped base: every rank computes the same offsets).
+size_t domain_bytes(const DomainBox &b, bool split) {
+  const int64_t nsx = (b.n[0] + 3 + 3) / 4 * 4, nnode = nsx * (b.n[1] + 3) * (b.n[2] + 3);
+  const int64_t zsx = (b.n[0] + 2 + 3) / 4 * 4, nzone = zsx * (b.n[1] + 2) * (b.n[2] + 2);
+  const size_t nb = align_up(nnode * sizeof(double), 256), zb = align_up(nzone * sizeof(double), 256);
+  return 12 * nb + 9 * zb + (split ? 24 * zb : 0);  // 12 node arrays, e x2, m, P, aux x5, [B x24]
+}
+
+void carve_views(void *base, const DomainBox &b, const int64_t N[3], int32_t dom, bool split,
+                 DomView view[2]) {
+  const int64_t n0 = b.n[0], n1 = b.n[1], n2 = b.n[2];
   // row pitches padded to 4 doubles (32 B): TMA needs 16-byte strides
   const int64_t nsx = (n0 + 3 + 3) / 4 * 4, nsxy = nsx * (n1 + 3), nnode = nsxy * (n2 + 3);
   const int64_t zsx = (n0 + 2 + 3) / 4 * 4, zsxy = zsx * (n1 + 2), nzone = zsxy * (n2 + 2);
-  if (nnode >= (int64_t(1) << 31))  // the cycle kernels index a domain's storage with int32
-    return set_err(h, HYDRO_EINVAL, "domain too large: split it into more domains (< 2^31 nodes)");
   const size_t nb = align_up(nnode * sizeof(double), 256), zb = align_up(nzone * sizeof(double), 256);
-  // 12 node arrays (2 parities x 6), e x2, m, P, aux x5, optional B x24
-  size_t bytes = 12 * nb + 9 * zb + (split ? 24 * zb : 0);
-  CK(cudaMalloc(&D.mem, bytes));
-  CK(cudaMemsetAsync(D.mem, 0, bytes, h->stream));
-  D.bytes = bytes;
-  char *p = (char *)D.mem;
+  char *p = (char *)base;
   double *nodes[12];
   for (int a = 0; a < 12; ++a, p += nb) nodes[a] = (double *)p;
   double *e0 = (double *)p; p += zb;
@@ -102,12 +111,12 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
   double *aux = (double *)p; p += 5 * zb;
   double *B = split ? (double *)p : nullptr;
   for (int par = 0; par < 2; ++par) {
-    DomView &v = D.view[par];
+    DomView &v = view[par];
     std::memset(&v, 0, sizeof(v));
     for (int a = 0; a < 3; ++a) {
-      v.lo[a] = D.box.lo[a];
-      v.n[a] = (int32_t)D.box.n[a];
-      v.N[a] = (int32_t)h->L.N[a];
+      v.lo[a] = b.lo[a];
+      v.n[a] = (int32_t)b.n[a];
+      v.N[a] = (int32_t)N[a];
     }
     v.nsx = nsx; v.nsxy = nsxy; v.zsx = zsx; v.zsxy = zsxy;
     v.nnode = nnode; v.nzone = zb / sizeof(double);  // zone array stride (aux/B planes)
@@ -117,8 +126,25 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
     v.e = par ? e1 : e0;
     v.en = par ? e0 : e1;
     v.m = m; v.P = P; v.B = B; v.aux = aux;
-    v.dom = D.dom;
+    v.dom = dom;
   }
+}
+
+}  // namespace hydro
+
+namespace {
+
+int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
+  const int64_t n0 = D.box.n[0], n1 = D.box.n[1], n2 = D.box.n[2];
+  const int64_t nsx = (n0 + 3 + 3) / 4 * 4, nsxy = nsx * (n1 + 3), nnode = nsxy * (n2 + 3);
+  const int64_t zsx = (n0 + 2 + 3) / 4 * 4, zsxy = zsx * (n1 + 2);
+  if (nnode >= (int64_t(1) << 31))  // the cycle kernels index a domain's storage with int32
+    return set_err(h, HYDRO_EINVAL, "domain too large: split it into more domains (< 2^31 nodes)");
+  const size_t bytes = domain_bytes(D.box, split);
+  CK(cudaMalloc(&D.mem, bytes));
+  CK(cudaMemsetAsync(D.mem, 0, bytes, h->stream));
+  D.bytes = bytes;
+  carve_views(D.mem, D.box, h->L.N, D.dom, split, D.view);
   // TMA descriptors (3-D tiled, fp64, box FUSED_BOX_X x (TY+3) x 1; out-of-bounds zero fill)
   static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
   if (!encode) {
@@ -264,7 +290,8 @@ int fold_finalize(const hydro_ctx *h) {
   (void)h;
   return 0;
 #endif
-  return (!h->split && h->doms.size() == 1 && !h->comm && h->n_local_pairs == 0) ? 1 : 0;
+  return (!h->split && h->doms.size() == 1 && !h->comm && !h->peer && h->n_local_pairs == 0) ? 1
+                                                                                           : 0;
 }
 
 void launch_node_stage(hydro_ctx *h, LocalDom &D, int par, cudaStream_t s) {
@@ -303,6 +330,10 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
   if (h->comm) {
     int rc = comm_halo(h->comm, par, s);
     if (rc) return set_err(h, rc, "halo exchange failed");
+  }
+  if (h->peer) {  // halo push into the peers + dt / error reduction through the mailboxes
+    int rc = peer_exchange(h->peer, h->views_dev[par], par, true, h->st, s);
+    if (rc) return set_err(h, rc, "peer exchange failed");
   }
   if (!fold_finalize(h)) launch_finalize(h->st, h->ph, s);
   CK(cudaGetLastError());
@@ -516,7 +547,10 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
            CK(cudaMemcpyAsync(h->local_pairs_dev, lp.data(), sizeof(HaloCopy) * lp.size(),
                               cudaMemcpyHostToDevice, h->stream));
          }
-         if (cfg->nranks > 1) {
+         if (cfg->nranks > 1 && (cfg->flags & HYDRO_FLAG_PEER)) {
+           int r = peer_create(&h->peer, cfg, &h->err);
+           if (r) return r;
+         } else if (cfg->nranks > 1) {
            int r = comm_create(&h->comm, cfg, h->L, remote, h->slot_of_dom, h->doms.empty() ? nullptr : nullptr,
                                h->stream, &h->err);
            if (r) return r;
@@ -543,8 +577,9 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
            int r = comm_dt_min(h->comm, &h->st->dtz_acc, h->stream);
            if (r) return set_err(h, r, "dt allreduce failed");
          }
-         launch_finalize_init(h->st, cfg->dt_first, cfg->dt_init, cfg->dt_max, cfg->t_stop,
-                              cfg->t0, h->stream);
+         if (!h->peer)  // peer transport: dt^0 is reduced over the ranks at hydro_peer_import
+           launch_finalize_init(h->st, cfg->dt_first, cfg->dt_init, cfg->dt_max, cfg->t_stop,
+                                cfg->t0, h->stream);
          CK(cudaGetLastError());
          CK(cudaStreamSynchronize(h->stream));
          return HYDRO_OK;
@@ -556,14 +591,46 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
     set_err(h, st, "initial mesh has a zone with volume <= 0");
     return fail(st);
   }
-  if (h->use_graph && (rc = build_graphs(h)) != HYDRO_OK) return fail(rc);
+  if (!h->peer && h->use_graph && (rc = build_graphs(h)) != HYDRO_OK) return fail(rc);
   *out = h;
+  return HYDRO_OK;
+}
+
+int hydro_peer_export(hydro_ctx *h, void *buf, size_t *len) {
+  if (!h || !len) return set_err(h, HYDRO_EINVAL, "NULL argument");
+  if (!h->peer) return set_err(h, HYDRO_EINVAL, "context not created with HYDRO_FLAG_PEER");
+  CK(cudaSetDevice(h->device));
+  std::vector<int32_t> doms;
+  std::vector<void *> bases;
+  for (LocalDom &D : h->doms) {
+    doms.push_back(D.dom);
+    bases.push_back(D.mem);
+  }
+  return peer_export(h->peer, doms, bases, buf, len, &h->err);
+}
+
+int hydro_peer_import(hydro_ctx *h, const void *all, size_t len_per_rank) {
+  if (!h || !all) return set_err(h, HYDRO_EINVAL, "NULL argument");
+  if (!h->peer) return set_err(h, HYDRO_EINVAL, "context not created with HYDRO_FLAG_PEER");
+  CK(cudaSetDevice(h->device));
+  int rc = peer_import(h->peer, h->L, h->slot_of_dom, h->split, all, len_per_rank, &h->err);
+  if (rc) return rc;
+  // dt^0 over all ranks (no halo: every rank initialised its ghosts from the global definition)
+  rc = peer_exchange(h->peer, h->views_dev[0], 0, false, h->st, h->stream);
+  if (rc) return set_err(h, rc, "peer dt^0 exchange failed");
+  launch_finalize_init(h->st, h->cfg.dt_first, h->cfg.dt_init, h->cfg.dt_max, h->cfg.t_stop,
+                       h->cfg.t0, h->stream);
+  CK(cudaGetLastError());
+  CK(cudaStreamSynchronize(h->stream));
+  if (h->use_graph && (rc = build_graphs(h)) != HYDRO_OK) return rc;
   return HYDRO_OK;
 }
 
 int hydro_step(hydro_ctx *h, int32_t ncycles, void *cuda_stream, hydro_info *info) {
   if (!h || ncycles < 0) return set_err(h, HYDRO_EINVAL, "bad argument");
   if (h->failed) return set_err(h, HYDRO_ESTATE, "context failed earlier");
+  if (h->peer && !peer_ready(h->peer))
+    return set_err(h, HYDRO_ESTATE, "peer transport: hydro_peer_import not called yet");
   CK(cudaSetDevice(h->device));
   cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : h->stream;
   for (int32_t c = 0; c < ncycles; ++c) {
@@ -695,12 +762,15 @@ int hydro_kernels_per_cycle(const hydro_ctx *h) {
   if (h->n_local_pairs > 0) k += 1;  // intra-GPU halo copy
   if (!fold_finalize(h)) k += 1;     // finalize
   if (h->comm) k += comm_kernels_per_cycle(h->comm);
+  if (h->peer) k += peer_kernels_per_cycle(h->peer);
   return k;
 }
 
 int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
   if (!h || ncycles <= 0 || !out_ms) return set_err(h, HYDRO_EINVAL, "bad argument");
   if (h->failed) return set_err(h, HYDRO_ESTATE, "context failed earlier");
+  if (h->peer && !peer_ready(h->peer))
+    return set_err(h, HYDRO_ESTATE, "peer transport: hydro_peer_import not called yet");
   CK(cudaSetDevice(h->device));
   cudaStream_t s = h->stream;
   cudaEvent_t ev[5];
@@ -727,6 +797,8 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
     CK(cudaEventRecord(ev[1], s));
     launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, h->halo_blocks, s);
     if (h->comm && comm_halo(h->comm, par, s)) return HYDRO_ENCCL;
+    if (h->peer && peer_exchange(h->peer, h->views_dev[par], par, true, h->st, s))
+      return HYDRO_ECUDA;
     CK(cudaEventRecord(ev[2], s));
     if (!fold_finalize(h)) launch_finalize(h->st, h->ph, s);
     CK(cudaEventRecord(ev[3], s));
@@ -769,6 +841,7 @@ int hydro_destroy(hydro_ctx *h) {
     if (h->views_dev[p]) cudaFree(h->views_dev[p]);
   }
   if (h->comm) comm_destroy(h->comm);
+  if (h->peer) peer_destroy(h->peer);
   for (LocalDom &D : h->doms)
     if (D.mem) cudaFree(D.mem);
   if (h->local_pairs_dev) cudaFree(h->local_pairs_dev);

@@ -25,6 +25,7 @@ ABI_VERSION = 1
 FLAG_NO_GRAPH = 1 << 0
 FLAG_SPLIT = 1 << 1
 FLAG_ONE_KERNEL = 1 << 2
+FLAG_PEER = 1 << 3
 
 STATUS = {0: "ok", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENCCL", -5: "ETANGLED",
           -6: "ENONFINITE", -7: "EDTMIN", -8: "ESTATE"}
@@ -92,6 +93,8 @@ def load_library(path: str = LIB_PATH) -> C.CDLL:
     L.hydro_weighted_slabs.argtypes = [C.c_int64, C.c_int32, C.POINTER(C.c_double),
                                        C.POINTER(C.c_int64)]
     L.hydro_comm_unique_id.argtypes = [C.c_void_p]
+    L.hydro_peer_export.argtypes = [C.c_void_p, C.c_void_p, C.POINTER(C.c_size_t)]
+    L.hydro_peer_import.argtypes = [C.c_void_p, C.c_void_p, C.c_size_t]
     L.hydro_time_kernels.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_double)]
     L.hydro_kernels_per_cycle.argtypes = [C.c_void_p]
     L.hydro_strerror.restype = C.c_char_p
@@ -136,6 +139,8 @@ class HydroConfig:
     path: str = "two"             # "two" (zone + node/energy kernels), "one" (one fused kernel),
                                   # "split" (plain 3-kernel pipeline, HYDRO_FLAG_SPLIT)
     graph: bool = True            # CUDA graphs (HYDRO_FLAG_NO_GRAPH when False)
+    transport: str = "nccl"       # nranks > 1: "nccl" (NCCL send/recv + allreduce) or "peer"
+                                  # (CUDA IPC peer stores + mailbox reduction; ranks may share a GPU)
 
 
 class HydroError(RuntimeError):
@@ -182,7 +187,8 @@ def _cfg_struct(cfg: HydroConfig, keep: list, comm_id: Optional[bytes] = None) -
         keep.append(buf)
         c.comm_id = C.cast(buf, C.c_void_p)
     c.flags = ((0 if cfg.graph else FLAG_NO_GRAPH) | (FLAG_SPLIT if cfg.path == "split" else 0)
-               | (FLAG_ONE_KERNEL if cfg.path == "one" else 0))
+               | (FLAG_ONE_KERNEL if cfg.path == "one" else 0)
+               | (FLAG_PEER if cfg.transport == "peer" else 0))
     return c
 
 
@@ -257,7 +263,7 @@ class Hydro:
         self._L = load_library()
         self._group = group
         comm_id = None
-        if cfg.nranks > 1:
+        if cfg.nranks > 1 and cfg.transport == "nccl":
             comm_id = self._bootstrap_comm_id()
         keep: list = []
         c = _cfg_struct(cfg, keep, comm_id)
@@ -266,6 +272,25 @@ class Hydro:
         if rc != 0:
             raise HydroError(rc, self._L.hydro_last_error(None).decode())
         self._h = h
+        if cfg.nranks > 1 and cfg.transport == "peer":
+            self._bootstrap_peers()
+
+    def _bootstrap_peers(self):
+        """HYDRO_FLAG_PEER: all-gather every rank's IPC handles, then hydro_peer_import."""
+        import torch.distributed as dist
+        n = C.c_size_t(0)
+        self._L.hydro_peer_export(self._h, None, C.byref(n))
+        buf = C.create_string_buffer(n.value)
+        rc = self._L.hydro_peer_export(self._h, buf, C.byref(n))
+        if rc != 0:
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+        recs = [None] * self.cfg.nranks
+        dist.all_gather_object(recs, bytes(buf.raw), group=self._group)
+        width = max(len(r) for r in recs)
+        allb = b"".join(r.ljust(width, b"\0") for r in recs)
+        rc = self._L.hydro_peer_import(self._h, allb, width)
+        if rc != 0:
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
 
     def _bootstrap_comm_id(self) -> bytes:
         import torch
