@@ -252,11 +252,15 @@ def main():
 
     ws, rank, local = dist_env()
     ngpu = max(ws, 1)
+    # HYDRO_SHARE_GPU=1 (testing only): every rank on device 0, gloo for the host collectives
+    share = os.environ.get("HYDRO_SHARE_GPU") == "1"
+    if share:
+        local = 0
     torch.cuda.set_device(local)
     dist = None
     if ws > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl")
+        dist.init_process_group("gloo" if share else "nccl")
     from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig
 
     kw, scaling, desc = workload(args.config, ngpu)
@@ -283,7 +287,7 @@ def main():
         torch.cuda.synchronize()
     ms = start.elapsed_time(end)
     if dist:
-        t = torch.tensor([ms], device="cuda")
+        t = torch.tensor([ms], device="cpu" if share else "cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
     barrier()
@@ -295,7 +299,7 @@ def main():
     kt = hyd.time_kernels(min(args.steps, 50))
     launches = hyd.kernels_per_cycle() * args.steps
     if dist:
-        t = torch.tensor([launches], device="cuda", dtype=torch.float64)
+        t = torch.tensor([launches], device="cpu" if share else "cuda", dtype=torch.float64)
         dist.all_reduce(t)
         launches = int(t.item())
 
