@@ -1,0 +1,14 @@
+"""Small runs of every cycle path for compute-sanitizer (memcheck / racecheck / synccheck)."""
+import sys
+from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig
+from paper_conf_icppw_pearce18_b200.inputs import jittered_state
+
+n = (40, 30, 20)
+cuts = [[0, 17, 40], [0, 12, 30], [0, 20]]
+for path in sys.argv[1:] or ["two", "one", "split"]:
+    kw = dict(n=n, ndom=(2, 2, 1), cuts=cuts, init="user", user=jittered_state(n, 3), path=path,
+              graph=False)
+    with Hydro(HydroConfig(**kw)) as h:
+        r = h.step(3)
+        f = h.fields(["e", "rho"])
+        print(path, r["status"], float(f["e"].sum()), flush=True)
