@@ -28,6 +28,8 @@ struct DomView {
   double *P;                            // split pipeline: zone P scratch
   double *B;                            // split pipeline: 24 corner-vector components per zone
   double *aux;                          // 5 zone arrays: rho, p, q, c, vol (get_fields)
+  double *mn8;                          // node: 8 / (sum of the <= 8 zone masses around it),
+                                        // constant (Lagrangian masses, S7); see k_nodal_mass
   int32_t dom;                          // global domain index
   int32_t pad_;
 

@@ -34,13 +34,17 @@ namespace {
 template <int TX, int TY>
 struct CTile {
   static constexpr int TXT = TX + 2, TYT = TY + 2;  // zone-stage tile (owned + 1 ring)
-  static constexpr int NZT = TXT * TYT;
+  // One row pitch PX for the threads, the node box and the zone box (TX + 3 node columns rounded
+  // up to a 16-byte TMA row): neighbour offsets are the same in every array and a warp's LDS.64
+  // over consecutive threads touches consecutive words (no bank conflicts at row wraps).
+  static constexpr int PX = FUSED_BOX_X;
+  static constexpr int NZT = PX * TYT;              // thread slots of the tile rows
   static constexpr int NTHR = (NZT + 31) / 32 * 32;
   static constexpr int ZS = NTHR;                   // zone-tile slots
   static constexpr int BXN = FUSED_BOX_X, BYN = TY + 3;  // TMA node box (x padded to 16 B)
   static constexpr int NN = BXN * BYN;
   static constexpr int RS = (NN + 15) / 16 * 16;    // stride of one node array (128 B aligned)
-  static constexpr int ZBX = TXT, ZBY = TYT;        // TMA zone box = the zone tile
+  static constexpr int ZBX = PX, ZBY = TYT;         // TMA zone box = the zone tile (+ pad)
   static constexpr int ZN = ZBX * ZBY;
   static constexpr int ZRS = (ZN + 15) / 16 * 16;
   // shared memory, in doubles; SoA everywhere so a warp's LDS.64 is conflict-free
@@ -49,14 +53,13 @@ struct CTile {
   static constexpr int OFF_XP = OFF_ZR + 9 * ZRS;   // [2 planes][3][RS] half-step positions
   static constexpr int OFF_G = OFF_XP + 6 * RS;     // [3 vectors][3][ZS] g_x, g_y, g_z
   static constexpr int OFF_UH = OFF_G + 9 * ZS;     // [3][ZS] u_half of node plane p
-  static constexpr int OFF_VS = OFF_UH + 3 * ZS;    // [3][ZS] u_half(p-1) + u_half(p)
-  static constexpr int OFF_P = OFF_VS + 3 * ZS;     // [ZS] P of zone plane p (FUSED)
+  static constexpr int OFF_P = OFF_UH + 3 * ZS;     // [ZS] P of zone plane p (FUSED)
   static constexpr int OFF_PS = OFF_P + ZS;         // [2][ZS] psi of x-low, y-low faces
   static constexpr int OFF_RED = OFF_PS + 2 * ZS;   // [32] block dt reduction
   static constexpr int OFF_BAR = OFF_RED + 32;      // 3 mbarriers
   static constexpr int TOTAL = OFF_BAR + 4;
   static constexpr size_t BYTES = sizeof(double) * TOTAL;
-  static_assert(BXN >= TX + 3, "TMA box too narrow");
+  static_assert(BXN >= TX + 3 && BXN == PX, "TMA box too narrow");
   static_assert(BYN <= 256 && BXN <= 256, "TMA box limit");
   static_assert((ZBX * 8) % 16 == 0, "TMA zone box rows must be 16-byte multiples");
   static_assert(ZRS >= ZS - 32 && ZN <= ZS, "zone tile fits the thread tile");
@@ -72,18 +75,20 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   extern __shared__ __align__(1024) double sm[];
   double *RAW = sm + T::OFF_RAW, *ZR = sm + T::OFF_ZR, *XP = sm + T::OFF_XP, *PSF = sm + T::OFF_P;
   double *GX = sm + T::OFF_G, *GY = GX + 3 * T::ZS, *GZ = GY + 3 * T::ZS;
-  double *UH = sm + T::OFF_UH, *VS = sm + T::OFF_VS, *PSX = sm + T::OFF_PS, *PSY = PSX + T::ZS;
+  double *UH = sm + T::OFF_UH, *PSX = sm + T::OFF_PS, *PSY = PSX + T::ZS;
   uint64_t *bar = reinterpret_cast<uint64_t *>(sm + T::OFF_BAR);
-  constexpr int ZS = T::ZS, RS = T::RS, TXT = T::TXT, ZRS = T::ZRS;
+  constexpr int ZS = T::ZS, RS = T::RS, TXT = T::TXT, ZRS = T::ZRS, PX = T::PX;
 
   const int t = threadIdx.x;
   const int i0 = blockIdx.x * TX, j0 = blockIdx.y * TY;
   const int k0 = blockIdx.z * KZ;
   const int k1 = min(k0 + KZ, d.n[2]);
   const int n0 = d.n[0], n1 = d.n[1], n2 = d.n[2];
-  const bool active = t < T::NZT;
-  const int tc = active ? t : T::NZT - 1;  // padding lanes shadow the last zone (never store)
-  const int tx = tc % TXT, ty = tc / TXT;
+  // lanes: zone/node (tx, ty) for tx < TXT; tx == TXT forms the box's last node column; the
+  // rest (tx == PX-1 and the padding warp's tail) form the box's last node row
+  const int tc = t;
+  const int tx = t % PX, ty = t / PX;
+  const bool active = t < T::NZT && tx < TXT;
   const int li = i0 - 1 + tx, lj = j0 - 1 + ty;  // local zone / node index of this thread
 
   if ((st->halted | st->done) != 0u) {  // no-op cycle: carry the state over to the next parity
@@ -130,21 +135,24 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   auto zraw = [&](int q) { return ZR + ((q - q0) % 3) * 3 * ZRS; };
   // X stage: half-step positions of node plane q into XP slot q&1.  Thread t forms its own
   // node (tx, ty) -- returned in registers -- and the box's last column / row are shared out.
-  const int nidx = ty * T::BXN + tx;  // this thread's node in the node box
+  const int nidx = t;  // this thread's node in the node box (pitch PX)
+  const bool xown = t < T::NZT && tx <= TXT;  // forms x_p of its own node
+  const int hrow = tx == PX - 1 ? ty : (t >= T::NZT ? T::TYT + (t - T::NZT) : -1);
+  constexpr int NHELP = T::TYT + (T::NTHR - T::NZT);  // lanes forming the last node row
   auto form_xp = [&](int q, double &px, double &py, double &pz) {
     const double *R = raw(q);
     double *X = XP + (q & 1) * 3 * RS;
     px = fma(hh, R[3 * RS + nidx], R[nidx]);
     py = fma(hh, R[4 * RS + nidx], R[RS + nidx]);
     pz = fma(hh, R[5 * RS + nidx], R[2 * RS + nidx]);
-    if (active) {
+    if (xown) {
       X[nidx] = px;
       X[RS + nidx] = py;
       X[2 * RS + nidx] = pz;
     }
-    // remaining nodes of the box: column TXT (rows 0..TYT) and row TYT (columns 0..TXT-1)
-    for (int e = t; e < T::TYT + 1 + TXT; e += T::NTHR) {
-      const int n = e <= T::TYT ? e * T::BXN + TXT : T::TYT * T::BXN + (e - T::TYT - 1);
+    // the box's last node row (TYT), columns 0..TXT
+    for (int e = hrow; e >= 0 && e <= TXT; e += NHELP) {
+      const int n = T::TYT * PX + e;
       X[n] = fma(hh, R[3 * RS + n], R[n]);
       X[RS + n] = fma(hh, R[4 * RS + n], R[RS + n]);
       X[2 * RS + n] = fma(hh, R[5 * RS + n], R[2 * RS + n]);
@@ -170,8 +178,9 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   // carried per-thread state
   double P_prev = 0.0, im_prev = 0.0, e_prev = 0.0;
   double axp = 0, ayp = 0, azp = 0, bxp = 0, byp = 0, bzp = 0;  // x-low / y-low faces, plane p-1
-  double Sx = 0, Sy = 0, Sz = 0, Msum_prev = 0;                   // in-plane node sums, plane p-1
+  double Sx = 0, Sy = 0, Sz = 0;                                  // in-plane node sums, plane p-1
   double uhp = 0, vhp = 0, whp = 0;                               // own u_half of plane p-1
+  double nxu = 0, nxv = 0, nxw = 0, nyu = 0, nyv = 0, nyw = 0;    // u_half of nodes x+1, y+1, p-1
   double psi_zlow = 0.0;
   double dt2min = INFINITY;
 
@@ -217,9 +226,11 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   __syncthreads();
 
   for (int p = k0 - 1; p <= k1; ++p) {
+    // 8 / nodal mass of this thread's node on plane p (read early: its latency hides under Z)
+    const double rinv_n = ((fl & F_NODE) && p >= k0) ? __ldg(d.mn8 + (p + 1) * nsxy + nrow) : 0.0;
     // ---------------------------------------------------------------- phase 1: E2(p-2), Z(p)
     if (p >= k0 + 2 && (fl & F_OWN)) {
-      const double Wk = 0.125 * e2_P * ((PSX[t + 1] + PSY[t + TXT]) + e2_part);
+      const double Wk = 0.125 * e2_P * ((PSX[t + 1] + PSY[t + PX]) + e2_part);
       d.en[(p - 1) * zsxy + zoff] = e2_e - dt * Wk * e2_im;
     }
     const bool exists = (fl & F_ZEX) && p >= gz_lo && p < gz_hi;
@@ -327,7 +338,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     if (FUSED) im = exists ? im : 0.0;
     // ---------------------------------------------------------------- G
     const double gxw = (tx > 0) ? 0.125 * (PS[tc - 1] - P) : 0.0;
-    const double gyw = (ty > 0) ? 0.125 * (PS[tc - TXT] - P) : 0.0;
+    const double gyw = (ty > 0) ? 0.125 * (PS[tc - PX] - P) : 0.0;
     const double gzw = 0.125 * (P_prev - P);
     const double gxx = gxw * ax0, gxy = gxw * ay0, gxz_ = gxw * az0;
     const double gyx = gyw * bx0, gyy = gyw * by0, gyz_ = gyw * bz0;
@@ -339,14 +350,13 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     // ---------------------------------------------------------------- N
     double uh = 0.0, vh = 0.0, wh = 0.0;
     if (fl & F_NODE) {
-      const int tn = tc - TXT;  // zone (tx, ty-1)
+      const int tn = tc - PX;  // zone (tx, ty-1)
       double a0, a1, a2_, b0, b1, b2;
       ld3(GX, tn, a0, a1, a2_);      // g_x of zone (tx, ty-1)
       ld3(GY, tc - 1, b0, b1, b2);   // g_y of zone (tx-1, ty)
       const double Cx = (gxx + a0) + (gyx + b0);
       const double Cy = (gxy + a1) + (gyy + b1);
       const double Cz = (gxz_ + a2_) + (gyz_ + b2);
-      const double Ms = (MS[tn - 1] + MS[tn]) + (MS[tc - 1] + m);
       if (p >= k0) {
         double c0, c1, c2_;
         ld3(GZ, tn - 1, a0, a1, a2_);
@@ -355,7 +365,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
         const double Fx = Sx + Cx + ((a0 + b0) + (c0 + gzx));
         const double Fy = Sy + Cy + ((a1 + b1) + (c1 + gzy));
         const double Fz = Sz + Cz + ((a2_ + b2) + (c2_ + gzz));
-        const double rinv = 8.0 * frcp(Msum_prev + Ms);
+        const double rinv = rinv_n;  // 8 / nodal mass (constant, d.mn8)
         const bool wall_z = p == wz_lo || p == wz_hi;
         const double axc = (fl & F_WX) ? 0.0 : Fx * rinv;
         const double ayc = (fl & F_WY) ? 0.0 : Fy * rinv;
@@ -366,19 +376,17 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
         vh = (v + vn) * 0.5;
         wh = (w + wn) * 0.5;
         st3(UH, tc, uh, vh, wh);
-        st3(VS, tc, uhp + uh, vhp + vh, whp + wh);
         if ((fl & F_NWR) && (p < k1 || p == n2)) {
           const int id = (p + 1) * nsxy + nrow;
-          d.xn[id] = Ra[nidx] + dt * uh;
-          d.yn[id] = Ra[RS + nidx] + dt * vh;
-          d.zn[id] = Ra[2 * RS + nidx] + dt * wh;
+          d.xn[id] = fma(hh, un, xpa);  // x + dt u_half = x_p + dt/2 u' (reading R21)
+          d.yn[id] = fma(hh, vn, ypa);
+          d.zn[id] = fma(hh, wn, zpa);
           d.un[id] = un;
           d.vn[id] = vn;
           d.wn[id] = wn;
         }
       }
       Sx = Cx; Sy = Cy; Sz = Cz;
-      Msum_prev = Ms;
     }
     __syncthreads();
     // ---------------------------------------------------------------- phase 3: X(p+2), E1(p-1)
@@ -391,26 +399,24 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     double psi_zhigh = 0.0, psx = 0.0, psy = 0.0;
     const double vsx = uhp + uh, vsy = vhp + vh, vsz = whp + wh;  // own two-plane u_half sum
     if (p >= k0) {
-      double a0, a1, a2_, b0, b1, b2, c0, c1, c2_;
+      // u_half of nodes (tx+1, ty) and (tx, ty+1) on plane p; with the values this thread read
+      // on plane p-1 (carried in registers) they give those nodes' two-plane sums
+      double a0 = 0, a1 = 0, a2_ = 0, b0 = 0, b1 = 0, b2 = 0, c0, c1, c2_;
+      if (fl & (F_EXY | F_EXZ)) ld3(UH, tc + 1, a0, a1, a2_);
+      if (fl & (F_EXX | F_EXZ)) ld3(UH, tc + PX, b0, b1, b2);
       if (p >= k0 + 1) {
-        if (fl & F_EXX) {  // x-low face of zone plane p-1: nodes (tx, ty..ty+1), planes p-1, p
-          ld3(VS, tc + TXT, a0, a1, a2_);
-          psx = axp * (vsx + a0) + ayp * (vsy + a1) + azp * (vsz + a2_);
-          PSX[t] = psx;
-        }
-        if (fl & F_EXY) {  // y-low face of zone plane p-1: nodes (tx..tx+1, ty), planes p-1, p
-          ld3(VS, tc + 1, a0, a1, a2_);
-          psy = bxp * (vsx + a0) + byp * (vsy + a1) + bzp * (vsz + a2_);
-          PSY[t] = psy;
-        }
+        if (fl & F_EXX)  // x-low face of zone plane p-1: nodes (tx, ty..ty+1), planes p-1, p
+          PSX[t] = psx = axp * (vsx + (nyu + b0)) + ayp * (vsy + (nyv + b1)) + azp * (vsz + (nyw + b2));
+        if (fl & F_EXY)  // y-low face of zone plane p-1: nodes (tx..tx+1, ty), planes p-1, p
+          PSY[t] = psy = bxp * (vsx + (nxu + a0)) + byp * (vsy + (nxv + a1)) + bzp * (vsz + (nxw + a2_));
       }
       if (fl & F_EXZ) {  // z-face at node plane p: nodes (tx..tx+1, ty..ty+1)
-        ld3(UH, tc + 1, a0, a1, a2_);
-        ld3(UH, tc + TXT, b0, b1, b2);
-        ld3(UH, tc + TXT + 1, c0, c1, c2_);
+        ld3(UH, tc + PX + 1, c0, c1, c2_);
         psi_zhigh = cx0 * ((uh + a0) + (b0 + c0)) + cy0 * ((vh + a1) + (b1 + c1)) +
                     cz0 * ((wh + a2_) + (b2 + c2_));
       }
+      nxu = a0; nxv = a1; nxw = a2_;
+      nyu = b0; nyv = b1; nyw = b2;
     }
     // E2 of zone plane p-1 runs in the next phase 1: W = P/8 (psi_xhi - psi_x + psi_yhi - psi_y
     // + psi_zhi - psi_zlo) with the high-face psi read from the neighbours
@@ -430,7 +436,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     xpb = xpc; ypb = ypc; zpb = zpc;
   }
   if (k1 >= k0 + 1 && (fl & F_OWN)) {  // the last pending E2 (zone plane k1-1)
-    const double Wk = 0.125 * e2_P * ((PSX[t + 1] + PSY[t + TXT]) + e2_part);
+    const double Wk = 0.125 * e2_P * ((PSX[t + 1] + PSY[t + PX]) + e2_part);
     d.en[k1 * zsxy + zoff] = e2_e - dt * Wk * e2_im;
   }
   if (FUSED) block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);

@@ -22,6 +22,9 @@ void launch_init_nodes(const DomView &d, const double origin[3], const double ex
 // 2 USER_MASS (m already in place, e already in place).
 void launch_init_zones(const DomView &d, int kind, double rho0, double e0, double E,
                        cudaStream_t s);
+// d.mn8 = 8 / sum of the zone masses around each node (nodes 0..n per axis; masses are fixed
+// after init, so once per run).
+void launch_nodal_mass(const DomView &d, cudaStream_t s);
 // dt^0 (S2-S6 at x^0 with no predictor) over owned zones -> st->dtz_acc, error flags.
 void launch_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 void launch_finalize_init(DevState *st, double dt_first, double dt_init, double dt_max,

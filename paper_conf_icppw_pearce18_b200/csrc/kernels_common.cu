@@ -87,6 +87,25 @@ __global__ void k_init_zones(DomView d, int kind, double rho0, double e0, double
   }
 }
 
+// Nodal inverse mass for the cycle kernels (S7: m_p = sum_z m_z / 8; zones outside the mesh have
+// m = 0).  Summed in the order the node stage used to sum it on the fly (x pairs, y pairs, then
+// the plane below + the plane above).
+__global__ void k_nodal_mass(DomView d) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int j = blockIdx.y * blockDim.y + threadIdx.y;
+  const int k = blockIdx.z;
+  if (i > d.n[0] || j > d.n[1]) return;
+  double ms[2];
+#pragma unroll
+  for (int c = 0; c < 2; ++c) {
+    const int kk = k - 1 + c;
+    ms[c] = (d.m[d.zid(i - 1, j - 1, kk)] + d.m[d.zid(i, j - 1, kk)]) +
+            (d.m[d.zid(i - 1, j, kk)] + d.m[d.zid(i, j, kk)]);
+  }
+  const double M = ms[0] + ms[1];
+  d.mn8[d.nid(i, j, k)] = M > 0.0 ? 8.0 / M : 0.0;
+}
+
 // dt^0: S2-S6 at x^0 with no predictor over owned zones.
 __global__ void k_dt0(DomView d, Phys ph, DevState *st) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
@@ -308,6 +327,9 @@ void launch_init_zones(const DomView &d, int kind, double rho0, double e0, doubl
                        cudaStream_t s) {
   k_init_zones<<<grid_for(d.n[0] + 2, d.n[1] + 2, d.n[2] + 2), dim3(BX, BY), 0, s>>>(
       d, kind, rho0, e0, E);
+}
+void launch_nodal_mass(const DomView &d, cudaStream_t s) {
+  k_nodal_mass<<<grid_for(d.n[0] + 1, d.n[1] + 1, d.n[2] + 1), dim3(BX, BY), 0, s>>>(d);
 }
 void launch_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
   k_dt0<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph, st);

@@ -91,7 +91,7 @@ size_t domain_bytes(const DomainBox &b, bool split) {
   const int64_t nsx = (b.n[0] + 3 + 3) / 4 * 4, nnode = nsx * (b.n[1] + 3) * (b.n[2] + 3);
   const int64_t zsx = (b.n[0] + 2 + 3) / 4 * 4, nzone = zsx * (b.n[1] + 2) * (b.n[2] + 2);
   const size_t nb = align_up(nnode * sizeof(double), 256), zb = align_up(nzone * sizeof(double), 256);
-  return 12 * nb + 9 * zb + (split ? 24 * zb : 0);  // 12 node arrays, e x2, m, P, aux x5, [B x24]
+  return 13 * nb + 9 * zb + (split ? 24 * zb : 0);  // 12 node arrays, mn8, e x2, m, P, aux x5, [B x24]
 }
 
 void carve_views(void *base, const DomainBox &b, const int64_t N[3], int32_t dom, bool split,
@@ -104,6 +104,7 @@ void carve_views(void *base, const DomainBox &b, const int64_t N[3], int32_t dom
   char *p = (char *)base;
   double *nodes[12];
   for (int a = 0; a < 12; ++a, p += nb) nodes[a] = (double *)p;
+  double *mn8 = (double *)p; p += nb;
   double *e0 = (double *)p; p += zb;
   double *e1 = (double *)p; p += zb;
   double *m = (double *)p; p += zb;
@@ -125,7 +126,7 @@ void carve_views(void *base, const DomainBox &b, const int64_t N[3], int32_t dom
     v.xn = nxt[0]; v.yn = nxt[1]; v.zn = nxt[2]; v.un = nxt[3]; v.vn = nxt[4]; v.wn = nxt[5];
     v.e = par ? e1 : e0;
     v.en = par ? e0 : e1;
-    v.m = m; v.P = P; v.B = B; v.aux = aux;
+    v.m = m; v.P = P; v.B = B; v.aux = aux; v.mn8 = mn8;
     v.dom = dom;
   }
 }
@@ -572,6 +573,7 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
          for (LocalDom &D : h->doms)
            launch_init_zones(D.view[0], cfg->init_kind, cfg->rho0, cfg->e0, cfg->sedov_energy,
                              h->stream);
+         for (LocalDom &D : h->doms) launch_nodal_mass(D.view[0], h->stream);
          for (LocalDom &D : h->doms) launch_dt0(D.view[0], h->ph, h->st, h->stream);
          if (h->comm) {
            int r = comm_dt_min(h->comm, &h->st->dtz_acc, h->stream);
