@@ -175,13 +175,21 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   }
   __syncthreads();
 
-  // carried per-thread state
-  double P_prev = 0.0, im_prev = 0.0, e_prev = 0.0;
-  double axp = 0, ayp = 0, azp = 0, bxp = 0, byp = 0, bzp = 0;  // x-low / y-low faces, plane p-1
-  double Sx = 0, Sy = 0, Sz = 0;                                  // in-plane node sums, plane p-1
-  double uhp = 0, vhp = 0, whp = 0;                               // own u_half of plane p-1
-  double nxu = 0, nxv = 0, nxw = 0, nyu = 0, nyv = 0, nyw = 0;    // u_half of nodes x+1, y+1, p-1
-  double psi_zlow = 0.0;
+  // Values one plane hands to the next.  Two sets alternate (the loop body runs twice per trip
+  // with the roles swapped), so nothing is copied between iterations: iteration p reads plane
+  // p-1's set `pv` and overwrites `cu`, which until then holds plane p-2 (the pending E2).
+  struct Carry {
+    double P, im, e;                // zone: P, 1/m, e
+    double ax, ay, az, bx, by, bz;  // zone: x-low and y-low face vectors
+    double Sx, Sy, Sz;              // node: sum of the 4 in-plane face forces of this zone plane
+    double uh, vh, wh;              // node: own u_half
+    double nxu, nxv, nxw;           // u_half of node (tx+1, ty)
+    double nyu, nyv, nyw;           // u_half of node (tx, ty+1)
+    double psiz;                    // psi of the z-face at this node plane
+    double part;                    // E2 partial sum of the zone plane (set one plane later)
+  };
+  struct XP3 { double x, y, z; };  // own node's half-step position
+  Carry S0 = {}, S1 = {};
   double dt2min = INFINITY;
 
   // Per-thread constants, kept in few registers (32-bit indices: a domain's storage is below
@@ -217,21 +225,20 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   //   phase 1: E2 of zone plane p-2 and the zone/face stage of plane p,
   //   phase 2: the node stage of node plane p,
   //   phase 3: x_p of node plane p+2 and E1 of zone plane p-1.
-  double xpa, ypa, zpa, xpb, ypb, zpb;  // own node's x_p at planes p and p+1
+  XP3 XA, XB;  // own node's x_p at planes p and p+1 (x_p of plane p+2 replaces plane p's)
   wait_plane(q0);
-  form_xp(q0, xpa, ypa, zpa);
+  form_xp(q0, XA.x, XA.y, XA.z);
   wait_plane(q0 + 1);
-  form_xp(q0 + 1, xpb, ypb, zpb);
-  double e2_P = 0.0, e2_e = 0.0, e2_im = 0.0, e2_part = 0.0;  // pending E2 of one zone plane
+  form_xp(q0 + 1, XB.x, XB.y, XB.z);
   __syncthreads();
 
-  for (int p = k0 - 1; p <= k1; ++p) {
+  auto body = [&](const int p, Carry &pv, Carry &cu, XP3 &xa, const XP3 &xb) {
     // 8 / nodal mass of this thread's node on plane p (read early: its latency hides under Z)
     const double rinv_n = ((fl & F_NODE) && p >= k0) ? __ldg(d.mn8 + (p + 1) * nsxy + nrow) : 0.0;
     // ---------------------------------------------------------------- phase 1: E2(p-2), Z(p)
-    if (p >= k0 + 2 && (fl & F_OWN)) {
-      const double Wk = 0.125 * e2_P * ((PSX[t + 1] + PSY[t + PX]) + e2_part);
-      d.en[(p - 1) * zsxy + zoff] = e2_e - dt * Wk * e2_im;
+    if (p >= k0 + 2 && (fl & F_OWN)) {  // cu still holds zone plane p-2
+      const double Wk = 0.125 * cu.P * ((PSX[t + 1] + PSY[t + PX]) + cu.part);
+      d.en[(p - 1) * zsxy + zoff] = cu.e - dt * Wk * cu.im;
     }
     const bool exists = (fl & F_ZEX) && p >= gz_lo && p < gz_hi;
     // zone plane p (TMA): m and e are 0 on zones outside the mesh (never written), P too
@@ -245,8 +252,8 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     if (FUSED) {
       const double *Rb = raw(p + 1);
       double X[8], Y[8], Z[8];
-      X[0] = xpa; Y[0] = ypa; Z[0] = zpa;
-      X[4] = xpb; Y[4] = ypb; Z[4] = zpb;
+      X[0] = xa.x; Y[0] = xa.y; Z[0] = xa.z;
+      X[4] = xb.x; Y[4] = xb.y; Z[4] = xb.z;
 #pragma unroll
       for (int l = 0; l < 8; ++l) {
         if (l == 0 || l == 4) continue;
@@ -321,8 +328,8 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
       __syncthreads();
     } else {
       double X[7], Y[7], Z[7];  // corners 0..6 (corner 7 lies on no low face)
-      X[0] = xpa; Y[0] = ypa; Z[0] = zpa;
-      X[4] = xpb; Y[4] = ypb; Z[4] = zpb;
+      X[0] = xa.x; Y[0] = xa.y; Z[0] = xa.z;
+      X[4] = xb.x; Y[4] = xb.y; Z[4] = xb.z;
 #pragma unroll
       for (int l = 1; l < 7; ++l) {
         if (l == 4) continue;
@@ -339,32 +346,34 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     // ---------------------------------------------------------------- G
     const double gxw = (tx > 0) ? 0.125 * (PS[tc - 1] - P) : 0.0;
     const double gyw = (ty > 0) ? 0.125 * (PS[tc - PX] - P) : 0.0;
-    const double gzw = 0.125 * (P_prev - P);
-    const double gxx = gxw * ax0, gxy = gxw * ay0, gxz_ = gxw * az0;
-    const double gyx = gyw * bx0, gyy = gyw * by0, gyz_ = gyw * bz0;
-    const double gzx = gzw * cx0, gzy = gzw * cy0, gzz = gzw * cz0;
-    st3(GX, t, gxx, gxy, gxz_);
-    st3(GY, t, gyx, gyy, gyz_);
-    st3(GZ, t, gzx, gzy, gzz);
+    const double gzw = 0.125 * (pv.P - P);
+    st3(GX, t, gxw * ax0, gxw * ay0, gxw * az0);
+    st3(GY, t, gyw * bx0, gyw * by0, gyw * bz0);
+    st3(GZ, t, gzw * cx0, gzw * cy0, gzw * cz0);
+    cu.P = P; cu.im = im; cu.e = e;
+    cu.ax = ax0; cu.ay = ay0; cu.az = az0;
+    cu.bx = bx0; cu.by = by0; cu.bz = bz0;
     __syncthreads();
     // ---------------------------------------------------------------- N
     double uh = 0.0, vh = 0.0, wh = 0.0;
+    double Cx = 0.0, Cy = 0.0, Cz = 0.0;
     if (fl & F_NODE) {
       const int tn = tc - PX;  // zone (tx, ty-1)
       double a0, a1, a2_, b0, b1, b2;
       ld3(GX, tn, a0, a1, a2_);      // g_x of zone (tx, ty-1)
       ld3(GY, tc - 1, b0, b1, b2);   // g_y of zone (tx-1, ty)
-      const double Cx = (gxx + a0) + (gyx + b0);
-      const double Cy = (gxy + a1) + (gyy + b1);
-      const double Cz = (gxz_ + a2_) + (gyz_ + b2);
+      // own faces' g enter fused (g = w A, not re-read): same value to within one rounding
+      Cx = fma(gxw, ax0, a0) + fma(gyw, bx0, b0);
+      Cy = fma(gxw, ay0, a1) + fma(gyw, by0, b1);
+      Cz = fma(gxw, az0, a2_) + fma(gyw, bz0, b2);
       if (p >= k0) {
         double c0, c1, c2_;
         ld3(GZ, tn - 1, a0, a1, a2_);
         ld3(GZ, tn, b0, b1, b2);
         ld3(GZ, tc - 1, c0, c1, c2_);
-        const double Fx = Sx + Cx + ((a0 + b0) + (c0 + gzx));
-        const double Fy = Sy + Cy + ((a1 + b1) + (c1 + gzy));
-        const double Fz = Sz + Cz + ((a2_ + b2) + (c2_ + gzz));
+        const double Fx = pv.Sx + Cx + ((a0 + b0) + fma(gzw, cx0, c0));
+        const double Fy = pv.Sy + Cy + ((a1 + b1) + fma(gzw, cy0, c1));
+        const double Fz = pv.Sz + Cz + ((a2_ + b2) + fma(gzw, cz0, c2_));
         const double rinv = rinv_n;  // 8 / nodal mass (constant, d.mn8)
         const bool wall_z = p == wz_lo || p == wz_hi;
         const double axc = (fl & F_WX) ? 0.0 : Fx * rinv;
@@ -378,66 +387,61 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
         st3(UH, tc, uh, vh, wh);
         if ((fl & F_NWR) && (p < k1 || p == n2)) {
           const int id = (p + 1) * nsxy + nrow;
-          d.xn[id] = fma(hh, un, xpa);  // x + dt u_half = x_p + dt/2 u' (reading R21)
-          d.yn[id] = fma(hh, vn, ypa);
-          d.zn[id] = fma(hh, wn, zpa);
+          d.xn[id] = fma(hh, un, xa.x);  // x + dt u_half = x_p + dt/2 u' (reading R21)
+          d.yn[id] = fma(hh, vn, xa.y);
+          d.zn[id] = fma(hh, wn, xa.z);
           d.un[id] = un;
           d.vn[id] = vn;
           d.wn[id] = wn;
         }
       }
-      Sx = Cx; Sy = Cy; Sz = Cz;
     }
+    cu.Sx = Cx; cu.Sy = Cy; cu.Sz = Cz;  // every set member is written every plane (short ranges)
+    cu.uh = uh; cu.vh = vh; cu.wh = wh;
     __syncthreads();
     // ---------------------------------------------------------------- phase 3: X(p+2), E1(p-1)
     if (t == 0 && p + 3 <= k1 + 1) issue(p + 3);  // slot of plane p, free after N(p)
-    double xpc = 0.0, ypc = 0.0, zpc = 0.0;
-    if (p + 2 <= k1 + 1) {
+    if (p + 2 <= k1 + 1) {  // x_p of plane p+2 into the registers of plane p (Z(p), N(p) done)
       wait_plane(p + 2);
-      form_xp(p + 2, xpc, ypc, zpc);
+      form_xp(p + 2, xa.x, xa.y, xa.z);
     }
-    double psi_zhigh = 0.0, psx = 0.0, psy = 0.0;
-    const double vsx = uhp + uh, vsy = vhp + vh, vsz = whp + wh;  // own two-plane u_half sum
-    if (p >= k0) {
-      // u_half of nodes (tx+1, ty) and (tx, ty+1) on plane p; with the values this thread read
-      // on plane p-1 (carried in registers) they give those nodes' two-plane sums
-      double a0 = 0, a1 = 0, a2_ = 0, b0 = 0, b1 = 0, b2 = 0, c0, c1, c2_;
-      if (fl & (F_EXY | F_EXZ)) ld3(UH, tc + 1, a0, a1, a2_);
-      if (fl & (F_EXX | F_EXZ)) ld3(UH, tc + PX, b0, b1, b2);
-      if (p >= k0 + 1) {
-        if (fl & F_EXX)  // x-low face of zone plane p-1: nodes (tx, ty..ty+1), planes p-1, p
-          PSX[t] = psx = axp * (vsx + (nyu + b0)) + ayp * (vsy + (nyv + b1)) + azp * (vsz + (nyw + b2));
-        if (fl & F_EXY)  // y-low face of zone plane p-1: nodes (tx..tx+1, ty), planes p-1, p
-          PSY[t] = psy = bxp * (vsx + (nxu + a0)) + byp * (vsy + (nxv + a1)) + bzp * (vsz + (nxw + a2_));
-      }
-      if (fl & F_EXZ) {  // z-face at node plane p: nodes (tx..tx+1, ty..ty+1)
-        ld3(UH, tc + PX + 1, c0, c1, c2_);
-        psi_zhigh = cx0 * ((uh + a0) + (b0 + c0)) + cy0 * ((vh + a1) + (b1 + c1)) +
-                    cz0 * ((wh + a2_) + (b2 + c2_));
-      }
-      nxu = a0; nxv = a1; nxw = a2_;
-      nyu = b0; nyv = b1; nyw = b2;
+    {
+      // E1 runs on every plane and lane (results of planes < k0+1 and of lanes whose faces do not
+      // matter are never read): u_half of nodes (tx+1, ty), (tx, ty+1), (tx+1, ty+1) on plane p;
+      // with the values of plane p-1 they give the neighbours' two-plane sums
+      const double vsx = pv.uh + uh, vsy = pv.vh + vh, vsz = pv.wh + wh;  // own two-plane sum
+      double a0, a1, a2_, b0, b1, b2, c0, c1, c2_;
+      ld3(UH, tc + 1, a0, a1, a2_);
+      ld3(UH, tc + PX, b0, b1, b2);
+      ld3(UH, tc + PX + 1, c0, c1, c2_);
+      // x-low face of zone plane p-1: nodes (tx, ty..ty+1), planes p-1, p
+      const double psx = pv.ax * (vsx + (pv.nyu + b0)) + pv.ay * (vsy + (pv.nyv + b1)) +
+                         pv.az * (vsz + (pv.nyw + b2));
+      // y-low face of zone plane p-1: nodes (tx..tx+1, ty), planes p-1, p
+      const double psy = pv.bx * (vsx + (pv.nxu + a0)) + pv.by * (vsy + (pv.nxv + a1)) +
+                         pv.bz * (vsz + (pv.nxw + a2_));
+      PSX[t] = psx;
+      PSY[t] = psy;
+      // z-face at node plane p: nodes (tx..tx+1, ty..ty+1)
+      const double psi_zhigh = cx0 * ((uh + a0) + (b0 + c0)) + cy0 * ((vh + a1) + (b1 + c1)) +
+                               cz0 * ((wh + a2_) + (b2 + c2_));
+      cu.nxu = a0; cu.nxv = a1; cu.nxw = a2_;
+      cu.nyu = b0; cu.nyv = b1; cu.nyw = b2;
+      // E2 of zone plane p-1 runs in the next phase 1: W = P/8 (psi_xhi - psi_x + psi_yhi - psi_y
+      // + psi_zhi - psi_zlo) with the high-face psi read from the neighbours
+      pv.part = ((psi_zhigh - pv.psiz) - psx) - psy;
+      cu.psiz = psi_zhigh;
     }
-    // E2 of zone plane p-1 runs in the next phase 1: W = P/8 (psi_xhi - psi_x + psi_yhi - psi_y
-    // + psi_zhi - psi_zlo) with the high-face psi read from the neighbours
-    e2_P = P_prev;
-    e2_e = e_prev;
-    e2_im = im_prev;
-    e2_part = ((psi_zhigh - psi_zlow) - psx) - psy;
     __syncthreads();
-    psi_zlow = psi_zhigh;
-    P_prev = P;
-    im_prev = im;
-    e_prev = e;
-    axp = ax0; ayp = ay0; azp = az0;
-    bxp = bx0; byp = by0; bzp = bz0;
-    uhp = uh; vhp = vh; whp = wh;
-    xpa = xpb; ypa = ypb; zpa = zpb;
-    xpb = xpc; ypb = ypc; zpb = zpc;
-  }
-  if (k1 >= k0 + 1 && (fl & F_OWN)) {  // the last pending E2 (zone plane k1-1)
-    const double Wk = 0.125 * e2_P * ((PSX[t + 1] + PSY[t + PX]) + e2_part);
-    d.en[k1 * zsxy + zoff] = e2_e - dt * Wk * e2_im;
+    if (p == k1 && k1 >= k0 + 1 && (fl & F_OWN)) {  // the last pending E2 (zone plane k1-1)
+      const double Wk = 0.125 * pv.P * ((PSX[t + 1] + PSY[t + PX]) + pv.part);
+      d.en[k1 * zsxy + zoff] = pv.e - dt * Wk * pv.im;
+    }
+  };
+  for (int p = k0 - 1; p <= k1; p += 2) {
+    body(p, S0, S1, XA, XB);
+    if (p + 1 > k1) break;
+    body(p + 1, S1, S0, XB, XA);
   }
   if (FUSED) block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);
   if (fold_finalize)  // single-domain, single-rank cycle: S9 here instead of a separate launch
