@@ -30,6 +30,7 @@ struct DomView {
   double *aux;                          // 5 zone arrays: rho, p, q, c, vol (get_fields)
   double *mn8;                          // node: 8 / (sum of the <= 8 zone masses around it),
                                         // constant (Lagrangian masses, S7); see k_nodal_mass
+  double *mi;                           // zone: 1 / m (0 outside the mesh), constant
   int32_t dom;                          // global domain index
   int32_t pad_;
 

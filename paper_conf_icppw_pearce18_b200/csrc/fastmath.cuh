@@ -2,8 +2,10 @@
 //
 // CUDA's IEEE fp64 division and sqrt carry a slow path (a call plus a reconvergence branch per
 // use); the fused kernel needs six of them per zone.  Here: the SFU seed (MUFU.RCP64H /
-// MUFU.RSQ64H) refined by Newton steps in DFMA, accurate to about 1 ulp, which the north_star
-// tolerance (1e-12 relative) absorbs (reading R12).
+// MUFU.RSQ64H) refined by Newton steps in DFMA.  Measured on B200 (tools/fastmath_acc.cu,
+// profiles/r01_fastmath_acc.txt, 2^28 log-uniform inputs over 2^-1000..2^1000): the seeds are
+// good to 2^-20, so two steps suffice -- rcp then matches IEEE 1/x exactly on every sample,
+// rsqrt is within 4e-16 relative -- which the north_star tolerance (1e-12) absorbs (reading R12).
 #pragma once
 
 namespace hydro {
@@ -14,8 +16,6 @@ __device__ __forceinline__ double frcp(double x) {  // 1/x for finite non-zero x
   double e = fma(-x, r, 1.0);
   r = fma(r, e, r);
   e = fma(-x, r, 1.0);
-  r = fma(r, e, r);
-  e = fma(-x, r, 1.0);
   return fma(r, e, r);
 }
 
@@ -23,7 +23,6 @@ __device__ __forceinline__ double frsqrt(double x) {  // 1/sqrt(x) for finite x 
   double y;
   asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
   const double h = 0.5 * x;
-  y = y * fma(-h * y, y, 1.5);
   y = y * fma(-h * y, y, 1.5);
   return y * fma(-h * y, y, 1.5);
 }

@@ -125,7 +125,8 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
 #pragma unroll
     for (int f = 0; f < 6; ++f) tma_load_3d(dst + f * RS, &maps.m[f], &bar[s], i0, j0, q + 1);
 #pragma unroll
-    for (int f = 0; f < NZF; ++f) tma_load_3d(zdst + f * ZRS, &maps.z[f], &bar[s], i0, j0, q + 1);
+    for (int f = 0; f < NZF; ++f)  // FUSED: m, e; else 1/m (z[3]), e, P
+      tma_load_3d(zdst + f * ZRS, &maps.z[(FUSED || f) ? f : 3], &bar[s], i0, j0, q + 1);
   };
   auto wait_plane = [&](int q) {
     const int u = q - q0;
@@ -340,7 +341,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
       HYDRO_FACE(X, Y, Z, 6, 0, 4, 2, ax0, ay0, az0);  // x-low (AX_0)
       HYDRO_FACE(X, Y, Z, 5, 0, 1, 4, bx0, by0, bz0);  // y-low (AY_0)
       HYDRO_FACE(X, Y, Z, 3, 0, 2, 1, cx0, cy0, cz0);  // z-low (AZ_0, node plane p)
-      im = exists ? frcp(m) : 0.0;
+      im = m;  // the ring's first field is 1/m here (0 outside the mesh)
     }
     if (FUSED) im = exists ? im : 0.0;
     // ---------------------------------------------------------------- G

@@ -106,21 +106,23 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
   double dt2min = INFINITY;
 
-  double m_nx = 0.0, e_nx = 0.0;
+  double m_nx = 0.0, e_nx = 0.0, mi_nx = 0.0;
   if (exists_xy && zk0 >= gz_lo && zk0 < gz_hi) {
     m_nx = d.m[(int64_t)(zk0 + 1) * d.zsxy + zrow];
     e_nx = d.e[(int64_t)(zk0 + 1) * d.zsxy + zrow];
+    mi_nx = d.mi[(int64_t)(zk0 + 1) * d.zsxy + zrow];
   }
 
   double zlx = 0.0, zly = 0.0, zlz = 0.0;  // z-high face of the zone below (carried)
   for (int p = zk0; p < zk1; ++p) {
-    const double m = m_nx, e = e_nx;
+    const double m = m_nx, e = e_nx, im = mi_nx;
     const bool exists = exists_xy && p >= gz_lo && p < gz_hi;
     {
       const int q = p + 1;
       const bool ok = q < zk1 && exists_xy && q >= gz_lo && q < gz_hi;
       m_nx = ok ? d.m[(int64_t)(q + 1) * d.zsxy + zrow] : 0.0;
       e_nx = ok ? d.e[(int64_t)(q + 1) * d.zsxy + zrow] : 0.0;
+      mi_nx = ok ? d.mi[(int64_t)(q + 1) * d.zsxy + zrow] : 0.0;
     }
     wait_plane(p + 1);
     form_xp(p + 1);
@@ -181,7 +183,6 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
     // S2-S4, S6 (see kernel_fused.cu for the algebra): L = 2V/sqrt(a2) enters through
     // s = -2 DV/sqrt(a2) and dt^2 = V^2 min(4 cfl^2/(a2 sigma^2), c_vol^2/DV^2).
     const double iV = frcp(V);
-    const double im = frcp(m);
     const double rho = m * iV;
     const double epos = e > 0.0 ? e : 0.0;
     const double ep = e - (hh * (ph.gm1 * rho) * epos) * DV * im;

@@ -22,6 +22,7 @@ void launch_init_nodes(const DomView &d, const double origin[3], const double ex
 // 2 USER_MASS (m already in place, e already in place).
 void launch_init_zones(const DomView &d, int kind, double rho0, double e0, double E,
                        cudaStream_t s);
+// d.mi = 1/m of every zone in storage (0 where m = 0) and
 // d.mn8 = 8 / sum of the zone masses around each node (nodes 0..n per axis; masses are fixed
 // after init, so once per run).
 void launch_nodal_mass(const DomView &d, cudaStream_t s);
@@ -39,7 +40,7 @@ void launch_energy_split(const DomView &d, const Phys &ph, DevState *st, cudaStr
 // zone arrays m, e, P (box = the kernel's zone tile).
 struct alignas(64) NodeMaps {
   CUtensorMap m[6];
-  CUtensorMap z[3];
+  CUtensorMap z[4];  // m, e, P, 1/m
 };
 
 // Fused single-kernel cycle (default path).

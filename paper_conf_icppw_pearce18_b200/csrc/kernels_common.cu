@@ -2,6 +2,7 @@
 // kernels, plus the split 3-kernel pipeline (zone / node / energy) that serves as the plain,
 // one-thread-per-element GPU path (HYDRO_FLAG_SPLIT).  The fused default path is in
 // kernel_fused.cu.
+#include <algorithm>
 #include <cmath>
 
 #include "kernels.h"
@@ -104,6 +105,14 @@ __global__ void k_nodal_mass(DomView d) {
   }
   const double M = ms[0] + ms[1];
   d.mn8[d.nid(i, j, k)] = M > 0.0 ? 8.0 / M : 0.0;
+}
+
+__global__ void k_inv_mass(DomView d, int64_t nz) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nz;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const double m = d.m[i];
+    d.mi[i] = m > 0.0 ? 1.0 / m : 0.0;
+  }
 }
 
 // dt^0: S2-S6 at x^0 with no predictor over owned zones.
@@ -329,6 +338,8 @@ void launch_init_zones(const DomView &d, int kind, double rho0, double e0, doubl
       d, kind, rho0, e0, E);
 }
 void launch_nodal_mass(const DomView &d, cudaStream_t s) {
+  const int64_t nz = d.zsxy * (d.n[2] + 2);
+  k_inv_mass<<<(int)std::min<int64_t>((nz + 255) / 256, 4096), 256, 0, s>>>(d, nz);
   k_nodal_mass<<<grid_for(d.n[0] + 1, d.n[1] + 1, d.n[2] + 1), dim3(BX, BY), 0, s>>>(d);
 }
 void launch_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {

@@ -91,7 +91,7 @@ size_t domain_bytes(const DomainBox &b, bool split) {
   const int64_t nsx = (b.n[0] + 3 + 3) / 4 * 4, nnode = nsx * (b.n[1] + 3) * (b.n[2] + 3);
   const int64_t zsx = (b.n[0] + 2 + 3) / 4 * 4, nzone = zsx * (b.n[1] + 2) * (b.n[2] + 2);
   const size_t nb = align_up(nnode * sizeof(double), 256), zb = align_up(nzone * sizeof(double), 256);
-  return 13 * nb + 9 * zb + (split ? 24 * zb : 0);  // 12 node arrays, mn8, e x2, m, P, aux x5, [B x24]
+  return 13 * nb + 10 * zb + (split ? 24 * zb : 0);  // 12 node arrays, mn8, e x2, m, mi, P, aux x5, [B x24]
 }
 
 void carve_views(void *base, const DomainBox &b, const int64_t N[3], int32_t dom, bool split,
@@ -108,6 +108,7 @@ void carve_views(void *base, const DomainBox &b, const int64_t N[3], int32_t dom
   double *e0 = (double *)p; p += zb;
   double *e1 = (double *)p; p += zb;
   double *m = (double *)p; p += zb;
+  double *mi = (double *)p; p += zb;
   double *P = (double *)p; p += zb;
   double *aux = (double *)p; p += 5 * zb;
   double *B = split ? (double *)p : nullptr;
@@ -126,7 +127,7 @@ void carve_views(void *base, const DomainBox &b, const int64_t N[3], int32_t dom
     v.xn = nxt[0]; v.yn = nxt[1]; v.zn = nxt[2]; v.un = nxt[3]; v.vn = nxt[4]; v.wn = nxt[5];
     v.e = par ? e1 : e0;
     v.en = par ? e0 : e1;
-    v.m = m; v.P = P; v.B = B; v.aux = aux; v.mn8 = mn8;
+    v.m = m; v.P = P; v.B = B; v.aux = aux; v.mn8 = mn8; v.mi = mi;
     v.dom = dom;
   }
 }
@@ -159,12 +160,12 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
   for (int par = 0; par < 2; ++par) {
     const double *arr[6] = {D.view[par].x, D.view[par].y, D.view[par].z,
                             D.view[par].u, D.view[par].v, D.view[par].w};
-    const double *zarr[3] = {D.view[par].m, D.view[par].e, D.view[par].P};
+    const double *zarr[4] = {D.view[par].m, D.view[par].e, D.view[par].P, D.view[par].mi};
     for (int kind = 0; kind < 2; ++kind) {
       if (kind == 0 && fused_box_y() != node_box_y())
         return set_err(h, HYDRO_EINVAL, "fused and node kernels must share a TMA box");
       NodeMaps &M = kind ? D.zmaps[par] : D.maps[par];
-      for (int f = 0; f < 9; ++f) {
+      for (int f = 0; f < 10; ++f) {
         const bool zf = f >= 6;
         const int64_t sx = zf ? zsx : nsx, sy = zf ? (n1 + 2) : (n1 + 3);
         const int64_t sz = zf ? (n2 + 2) : (n2 + 3), sxy = zf ? zsxy : nsxy;
