@@ -101,28 +101,32 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   const bool exists_xy = in_xy && gx >= 0 && gx < d.N[0] && gy >= 0 && gy < d.N[1];
   const bool owned_xy = li >= 0 && lj >= 0 && li < n0 && lj < n1;
   const int nidx = ty * ZNX + tx + xoff;
-  const int64_t zrow = (int64_t)(lj + 1) * d.zsx + (li + 1);
-  const int64_t gz_lo = -d.lo[2], gz_hi = d.N[2] - d.lo[2];
+  // 32-bit storage indices (a domain's storage is below 2^31 elements, checked at create)
+  const int zrow = (lj + 1) * (int)d.zsx + (li + 1), zsxy = (int)d.zsxy;
+  const int gz_lo = -(int)d.lo[2], gz_hi = d.N[2] - (int)d.lo[2];
   const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
   double dt2min = INFINITY;
 
-  double m_nx = 0.0, e_nx = 0.0, mi_nx = 0.0;
+  // Values handed from plane p to plane p+1: the zone's m, e, 1/m (prefetched one plane ahead)
+  // and its z-high face (= the z-low face of the zone above).  Two sets alternate (the body runs
+  // twice per trip with the roles swapped), so no registers are copied between planes.
+  struct Carry { double m, e, mi, zx, zy, zz, za2; };
+  Carry S0 = {}, S1 = {};
   if (exists_xy && zk0 >= gz_lo && zk0 < gz_hi) {
-    m_nx = d.m[(int64_t)(zk0 + 1) * d.zsxy + zrow];
-    e_nx = d.e[(int64_t)(zk0 + 1) * d.zsxy + zrow];
-    mi_nx = d.mi[(int64_t)(zk0 + 1) * d.zsxy + zrow];
+    S0.m = d.m[(zk0 + 1) * zsxy + zrow];
+    S0.e = d.e[(zk0 + 1) * zsxy + zrow];
+    S0.mi = d.mi[(zk0 + 1) * zsxy + zrow];
   }
 
-  double zlx = 0.0, zly = 0.0, zlz = 0.0;  // z-high face of the zone below (carried)
-  for (int p = zk0; p < zk1; ++p) {
-    const double m = m_nx, e = e_nx, im = mi_nx;
+  auto body = [&](const int p, const Carry &cu, Carry &nx) {
+    const double m = cu.m, e = cu.e, im = cu.mi;
     const bool exists = exists_xy && p >= gz_lo && p < gz_hi;
     {
       const int q = p + 1;
       const bool ok = q < zk1 && exists_xy && q >= gz_lo && q < gz_hi;
-      m_nx = ok ? d.m[(int64_t)(q + 1) * d.zsxy + zrow] : 0.0;
-      e_nx = ok ? d.e[(int64_t)(q + 1) * d.zsxy + zrow] : 0.0;
-      mi_nx = ok ? d.mi[(int64_t)(q + 1) * d.zsxy + zrow] : 0.0;
+      nx.m = ok ? d.m[(q + 1) * zsxy + zrow] : 0.0;
+      nx.e = ok ? d.e[(q + 1) * zsxy + zrow] : 0.0;
+      nx.mi = ok ? d.mi[(q + 1) * zsxy + zrow] : 0.0;
     }
     wait_plane(p + 1);
     form_xp(p + 1);
@@ -147,10 +151,15 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
     for (int b = 0; b < 2; ++b)
       HYDRO_FACE(X, Y, Z, 5 + 2 * b, 2 * b, 1 + 2 * b, 2 * b + 4, fx[2 + b], fy[2 + b], fz[2 + b]);
     // z-low face = the z-high face this thread formed for the zone below (same nodes, same bits)
-    if (p == zk0) HYDRO_FACE(X, Y, Z, 3, 0, 2, 1, zlx, zly, zlz);
-    fx[4] = zlx; fy[4] = zly; fz[4] = zlz;
+    double za2 = cu.za2;
+    if (p == zk0) {
+      HYDRO_FACE(X, Y, Z, 3, 0, 2, 1, fx[4], fy[4], fz[4]);
+      za2 = fx[4] * fx[4] + fy[4] * fy[4] + fz[4] * fz[4];
+    } else {
+      fx[4] = cu.zx; fy[4] = cu.zy; fz[4] = cu.zz;
+    }
     HYDRO_FACE(X, Y, Z, 7, 4, 6, 5, fx[5], fy[5], fz[5]);
-    zlx = fx[5]; zly = fy[5]; zlz = fz[5];
+    nx.zx = fx[5]; nx.zy = fy[5]; nx.zz = fz[5];
     // corner vectors S_l = s(a)AX_a + (s(b)AY_b + s(c)AZ_c): the (b, c) pair sums once
     double qx[4], qy[4], qz[4];
 #pragma unroll
@@ -174,13 +183,17 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
     }
     const double V = V8 * (1.0 / 24.0);
     const double DV = 0.125 * DV8;
-    double a2 = fx[0] * fx[0] + fy[0] * fy[0] + fz[0] * fz[0];
+    // max squared face area; the z-high face's square is handed to the zone above
+    const double zh2 = fx[5] * fx[5] + fy[5] * fy[5] + fz[5] * fz[5];
+    nx.za2 = zh2;
+    // (compare-select, not fmax: fp64 fmax costs a NaN-handling sequence; the areas are finite)
+    double a2 = zh2 > za2 ? zh2 : za2;
 #pragma unroll
-    for (int f = 1; f < 6; ++f) {
+    for (int f = 0; f < 4; ++f) {
       const double v = fx[f] * fx[f] + fy[f] * fy[f] + fz[f] * fz[f];
       a2 = v > a2 ? v : a2;
     }
-    // S2-S4, S6 (see kernel_fused.cu for the algebra): L = 2V/sqrt(a2) enters through
+    // S2-S4, S6 (see kernel_cycle.cu for the algebra): L = 2V/sqrt(a2) enters through
     // s = -2 DV/sqrt(a2) and dt^2 = V^2 min(4 cfl^2/(a2 sigma^2), c_vol^2/DV^2).
     const double iV = frcp(V);
     const double rho = m * iV;
@@ -196,7 +209,7 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
       qr = s * (ph.q_quad * s + ph.q_lin * c);
     }
     const double P = exists ? pr + rho * qr : 0.0;
-    if (in_xy) d.P[(int64_t)(p + 1) * d.zsxy + zrow] = P;
+    if (in_xy) d.P[(p + 1) * zsxy + zrow] = P;
     if (exists && owned_xy && p >= 0 && p < n2) {
       const double V2 = V * V;
       const double n1c = cfl4 * V2, d1c = (c2 + 2.0 * qr) * a2;
@@ -211,6 +224,11 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
         flag_error_zone(st, (V > 0.0) ? ERR_NONFINITE : ERR_TANGLED, gzi);
       }
     }
+  };
+  for (int p = zk0; p < zk1; p += 2) {
+    body(p, S0, S1);
+    if (p + 1 >= zk1) break;
+    body(p + 1, S1, S0);
   }
   block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + ZOFF_RED);
 }
