@@ -265,14 +265,18 @@ __global__ void k_halo_copy(const DomView *views, const HaloCopy *pairs) {
   const HaloCopy p = pairs[blockIdx.y];
   const DomView &D = views[p.dst];
   const DomView &S = views[p.src];
-  const int64_t nx = p.nhi[0] - p.nlo[0], ny = p.nhi[1] - p.nlo[1], nz = p.nhi[2] - p.nlo[2];
-  const int64_t nn = nx * ny * nz;
-  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nn;
-       t += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t a = t % nx, b = (t / nx) % ny, c = t / (nx * ny);
-    const int64_t gx = p.nlo[0] + a, gy = p.nlo[1] + b, gz = p.nlo[2] + c;
-    const int64_t di = D.nid((int)(gx - D.lo[0]), (int)(gy - D.lo[1]), (int)(gz - D.lo[2]));
-    const int64_t si = S.nid((int)(gx - S.lo[0]), (int)(gy - S.lo[1]), (int)(gz - S.lo[2]));
+  // 32-bit index arithmetic (slabs and domain storage are below 2^31 elements)
+  const int nx = (int)(p.nhi[0] - p.nlo[0]), ny = (int)(p.nhi[1] - p.nlo[1]);
+  const int nn = nx * ny * (int)(p.nhi[2] - p.nlo[2]);
+  // local node index of the slab origin in both domains; element (a, b, c) is origin + offsets
+  const int dsx = (int)D.nsx, dsxy = (int)D.nsxy, ssx = (int)S.nsx, ssxy = (int)S.nsxy;
+  const int d0 = (int)D.nid((int)(p.nlo[0] - D.lo[0]), (int)(p.nlo[1] - D.lo[1]),
+                            (int)(p.nlo[2] - D.lo[2]));
+  const int s0 = (int)S.nid((int)(p.nlo[0] - S.lo[0]), (int)(p.nlo[1] - S.lo[1]),
+                            (int)(p.nlo[2] - S.lo[2]));
+  for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < nn; t += gridDim.x * blockDim.x) {
+    const int a = t % nx, r = t / nx, b = r % ny, c = r / ny;
+    const int di = d0 + c * dsxy + b * dsx + a, si = s0 + c * ssxy + b * ssx + a;
     D.xn[di] = S.xn[si];
     D.yn[di] = S.yn[si];
     D.zn[di] = S.zn[si];
@@ -280,14 +284,16 @@ __global__ void k_halo_copy(const DomView *views, const HaloCopy *pairs) {
     D.vn[di] = S.vn[si];
     D.wn[di] = S.wn[si];
   }
-  const int64_t zx = p.zhi[0] - p.zlo[0], zy = p.zhi[1] - p.zlo[1], zz = p.zhi[2] - p.zlo[2];
-  const int64_t nzn = zx * zy * zz;
-  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nzn;
-       t += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t a = t % zx, b = (t / zx) % zy, c = t / (zx * zy);
-    const int64_t gx = p.zlo[0] + a, gy = p.zlo[1] + b, gz = p.zlo[2] + c;
-    D.en[D.zid((int)(gx - D.lo[0]), (int)(gy - D.lo[1]), (int)(gz - D.lo[2]))] =
-        S.en[S.zid((int)(gx - S.lo[0]), (int)(gy - S.lo[1]), (int)(gz - S.lo[2]))];
+  const int zx = (int)(p.zhi[0] - p.zlo[0]), zy = (int)(p.zhi[1] - p.zlo[1]);
+  const int nzn = zx * zy * (int)(p.zhi[2] - p.zlo[2]);
+  const int zdsx = (int)D.zsx, zdsxy = (int)D.zsxy, zssx = (int)S.zsx, zssxy = (int)S.zsxy;
+  const int zd0 = (int)D.zid((int)(p.zlo[0] - D.lo[0]), (int)(p.zlo[1] - D.lo[1]),
+                             (int)(p.zlo[2] - D.lo[2]));
+  const int zs0 = (int)S.zid((int)(p.zlo[0] - S.lo[0]), (int)(p.zlo[1] - S.lo[1]),
+                             (int)(p.zlo[2] - S.lo[2]));
+  for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < nzn; t += gridDim.x * blockDim.x) {
+    const int a = t % zx, r = t / zx, b = r % zy, c = r / zy;
+    D.en[zd0 + c * zdsxy + b * zdsx + a] = S.en[zs0 + c * zssxy + b * zssx + a];
   }
 }
 
