@@ -56,8 +56,8 @@ struct CTile {
   static constexpr int OFF_P = OFF_UH + 3 * ZS;     // [ZS] P of zone plane p (FUSED)
   static constexpr int OFF_PS = OFF_P + ZS;         // [2][ZS] psi of x-low, y-low faces
   static constexpr int OFF_RED = OFF_PS + 2 * ZS;   // [32] block dt reduction
-  static constexpr int OFF_BAR = OFF_RED + 32;      // 3 mbarriers
-  static constexpr int TOTAL = OFF_BAR + 4;
+  static constexpr int OFF_BAR = OFF_RED + 32;      // 3 TMA mbarriers + 3 phase mbarriers
+  static constexpr int TOTAL = OFF_BAR + 8;
   static constexpr size_t BYTES = sizeof(double) * TOTAL;
   static_assert(BXN >= TX + 3 && BXN == PX, "TMA box too narrow");
   static_assert(BYN <= 256 && BXN <= 256, "TMA box limit");
@@ -169,6 +169,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   if (t == 0) {
     if (smem_u32(sm) & 127u) __trap();  // TMA destinations must be 128-byte aligned
     for (int s = 0; s < 3; ++s) mbar_init(&bar[s], 1);
+    for (int s = 3; s < 6; ++s) mbar_init(&bar[s], T::NTHR / 32);  // one arrival per warp
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     issue(q0);
     issue(q0 + 1);
@@ -233,14 +234,27 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   form_xp(q0 + 1, XB.x, XB.y, XB.z);
   __syncthreads();
 
+  // Split phase barriers (node/energy kernel): a warp arrives once its shared-memory writes of a
+  // phase are done, runs work that does not read them, then waits.  Every barrier completes once
+  // per plane, so plane p waits on parity (p - q0) & 1.  The fused kernel uses __syncthreads.
+  enum { B_G = 3, B_U = 4, B_P = 5 };
+  auto arrive = [&](int b) {
+    __syncwarp();
+    if ((t & 31) == 0) mbar_arrive(&bar[b]);
+  };
+  auto await = [&](int b, int p) { mbar_wait(&bar[b], (uint32_t)((p - q0) & 1)); };
+  auto energy2 = [&](int zp, const Carry &c) {  // E2 of zone plane zp from its carry set
+    if (fl & F_OWN) {
+      const double Wk = 0.125 * c.P * ((PSX[t + 1] + PSY[t + PX]) + c.part);
+      d.en[(zp + 1) * zsxy + zoff] = c.e - dt * Wk * c.im;
+    }
+  };
+
   auto body = [&](const int p, Carry &pv, Carry &cu, XP3 &xa, const XP3 &xb) {
     // 8 / nodal mass of this thread's node on plane p (read early: its latency hides under Z)
     const double rinv_n = ((fl & F_NODE) && p >= k0) ? __ldg(d.mn8 + (p + 1) * nsxy + nrow) : 0.0;
     // ---------------------------------------------------------------- phase 1: E2(p-2), Z(p)
-    if (p >= k0 + 2 && (fl & F_OWN)) {  // cu still holds zone plane p-2
-      const double Wk = 0.125 * cu.P * ((PSX[t + 1] + PSY[t + PX]) + cu.part);
-      d.en[(p - 1) * zsxy + zoff] = cu.e - dt * Wk * cu.im;
-    }
+    if (FUSED && p >= k0 + 2) energy2(p - 2, cu);  // cu still holds zone plane p-2
     const bool exists = (fl & F_ZEX) && p >= gz_lo && p < gz_hi;
     // zone plane p (TMA): m and e are 0 on zones outside the mesh (never written), P too
     double *MS = zraw(p), *ES = MS + ZRS, *PS = FUSED ? PSF : MS + 2 * ZRS;
@@ -248,6 +262,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     double P = FUSED ? 0.0 : PS[tc];
     const double *Ra = raw(p);
     const double *Xa = XP + (p & 1) * 3 * RS, *Xb = XP + ((p + 1) & 1) * 3 * RS;
+    if (!FUSED && p > q0) await(B_P, p - 1);  // x_p(p+1) and psi of the previous plane
     double im;
     double ax0, ay0, az0, bx0, by0, bz0, cx0, cy0, cz0;
     if (FUSED) {
@@ -351,10 +366,16 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     st3(GX, t, gxw * ax0, gxw * ay0, gxw * az0);
     st3(GY, t, gyw * bx0, gyw * by0, gyw * bz0);
     st3(GZ, t, gzw * cx0, gzw * cy0, gzw * cz0);
+    if (FUSED) {
+      __syncthreads();
+    } else {
+      arrive(B_G);
+      if (p >= k0 + 2) energy2(p - 2, cu);  // cu still holds zone plane p-2
+      await(B_G, p);
+    }
     cu.P = P; cu.im = im; cu.e = e;
     cu.ax = ax0; cu.ay = ay0; cu.az = az0;
     cu.bx = bx0; cu.by = by0; cu.bz = bz0;
-    __syncthreads();
     // ---------------------------------------------------------------- N
     double uh = 0.0, vh = 0.0, wh = 0.0;
     double Cx = 0.0, Cy = 0.0, Cz = 0.0;
@@ -399,12 +420,20 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     }
     cu.Sx = Cx; cu.Sy = Cy; cu.Sz = Cz;  // every set member is written every plane (short ranges)
     cu.uh = uh; cu.vh = vh; cu.wh = wh;
-    __syncthreads();
     // ---------------------------------------------------------------- phase 3: X(p+2), E1(p-1)
-    if (t == 0 && p + 3 <= k1 + 1) issue(p + 3);  // slot of plane p, free after N(p)
-    if (p + 2 <= k1 + 1) {  // x_p of plane p+2 into the registers of plane p (Z(p), N(p) done)
+    if (FUSED) {
+      __syncthreads();
+      if (t == 0 && p + 3 <= k1 + 1) issue(p + 3);  // slot of plane p, free after N(p)
+    } else {
+      arrive(B_U);
+    }
+    if (p + 2 <= k1 + 1) {  // x_p of plane p+2 into the registers of plane p (Z(p) done)
       wait_plane(p + 2);
       form_xp(p + 2, xa.x, xa.y, xa.z);
+    }
+    if (!FUSED) {
+      await(B_U, p);
+      if (t == 0 && p + 3 <= k1 + 1) issue(p + 3);  // slot of plane p, free after N(p)
     }
     {
       // E1 runs on every plane and lane (results of planes < k0+1 and of lanes whose faces do not
@@ -433,10 +462,11 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
       pv.part = ((psi_zhigh - pv.psiz) - psx) - psy;
       cu.psiz = psi_zhigh;
     }
-    __syncthreads();
-    if (p == k1 && k1 >= k0 + 1 && (fl & F_OWN)) {  // the last pending E2 (zone plane k1-1)
-      const double Wk = 0.125 * pv.P * ((PSX[t + 1] + PSY[t + PX]) + pv.part);
-      d.en[k1 * zsxy + zoff] = pv.e - dt * Wk * pv.im;
+    if (FUSED) __syncthreads();
+    else arrive(B_P);
+    if (p == k1 && k1 >= k0 + 1) {  // the last pending E2 (zone plane k1-1)
+      if (!FUSED) await(B_P, p);
+      energy2(k1 - 1, pv);
     }
   };
   for (int p = k0 - 1; p <= k1; p += 2) {
