@@ -29,10 +29,11 @@ constexpr int ZBX = 32, ZBY = 8;                       // zones per block (x, y)
 constexpr int ZNX = ZONE_BOX_X, ZNY = ZBY + 1;         // TMA node box (x padded to 16 B)
 constexpr int ZNN = ZNX * ZNY;
 constexpr int ZRS = (ZNN + 15) / 16 * 16;              // stride of one node array (128 B)
-constexpr int ZOFF_RAW = 0;                            // [3 slots][6 fields][ZRS]
-constexpr int ZOFF_XP = ZOFF_RAW + 18 * ZRS;           // [3 slots][3][ZRS]
+constexpr int ZRING = 4;                               // TMA ring: planes issued 3 ahead
+constexpr int ZOFF_RAW = 0;                            // [ZRING slots][6 fields][ZRS]
+constexpr int ZOFF_XP = ZOFF_RAW + ZRING * 6 * ZRS;    // [3 slots][3][ZRS]
 constexpr int ZOFF_RED = ZOFF_XP + 9 * ZRS;            // [32]
-constexpr int ZOFF_BAR = ZOFF_RED + 32;                // 3 mbarriers
+constexpr int ZOFF_BAR = ZOFF_RED + 32;                // ZRING mbarriers
 constexpr int ZTOTAL = ZOFF_BAR + 4;
 constexpr size_t ZBYTES = ZTOTAL * sizeof(double);
 static_assert(ZNX >= ZBX + 2, "zone-kernel TMA box too narrow (33 nodes + 1 alignment shift)");
@@ -62,10 +63,10 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   const double dt = st->dt;
   const double hh = 0.5 * dt;
 
-  // node plane q (local) -> slot (q - zk0) % 3; storage coordinates of the box origin
+  // node plane q (local) -> slot (q - zk0) % ZRING; storage coordinates of the box origin
   auto issue = [&](int q) {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    const int s = (q - zk0) % 3;
+    const int s = (q - zk0) % ZRING;
     double *dst = RAW + s * 6 * ZRS;
     mbar_expect_tx(&bar[s], 6u * ZNN * sizeof(double));
 #pragma unroll
@@ -73,10 +74,10 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   };
   auto wait_plane = [&](int q) {
     const int u = q - zk0;
-    mbar_wait(&bar[u % 3], (uint32_t)((u / 3) & 1));
+    mbar_wait(&bar[u % ZRING], (uint32_t)((u / ZRING) & 1));
   };
   auto form_xp = [&](int q) {
-    const double *R = RAW + ((q - zk0) % 3) * 6 * ZRS;
+    const double *R = RAW + ((q - zk0) % ZRING) * 6 * ZRS;
     double *X = XP + ((q - zk0) % 3) * 3 * ZRS;
     for (int n = t; n < ZNN; n += ZBX * ZBY) {
       X[n] = fma(hh, R[3 * ZRS + n], R[n]);
@@ -87,10 +88,9 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
 
   if (t == 0) {
     if (smem_u32(sm) & 127u) __trap();
-    for (int s = 0; s < 3; ++s) mbar_init(&bar[s], 1);
+    for (int s = 0; s < ZRING; ++s) mbar_init(&bar[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    issue(zk0);
-    issue(zk0 + 1);
+    for (int q = zk0; q < zk0 + ZRING - 1 && q <= zk1; ++q) issue(q);
   }
   __syncthreads();
   wait_plane(zk0);
@@ -131,10 +131,10 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
     wait_plane(p + 1);
     form_xp(p + 1);
     __syncthreads();
-    if (t == 0 && p + 2 <= zk1) issue(p + 2);  // into the slot of plane p-1 (no longer read)
+    if (t == 0 && p + ZRING - 1 <= zk1) issue(p + ZRING - 1);  // slot of plane p-1 (no longer read)
     const double *Xa = XP + ((p - zk0) % 3) * 3 * ZRS, *Xb = XP + ((p + 1 - zk0) % 3) * 3 * ZRS;
-    const double *Ua = RAW + ((p - zk0) % 3) * 6 * ZRS + 3 * ZRS;
-    const double *Ub = RAW + ((p + 1 - zk0) % 3) * 6 * ZRS + 3 * ZRS;
+    const double *Ua = RAW + ((p - zk0) % ZRING) * 6 * ZRS + 3 * ZRS;
+    const double *Ub = RAW + ((p + 1 - zk0) % ZRING) * 6 * ZRS + 3 * ZRS;
     double X[8], Y[8], Z[8];
 #pragma unroll
     for (int l = 0; l < 8; ++l) {
