@@ -48,8 +48,12 @@ struct CTile {
   static constexpr int ZN = ZBX * ZBY;
   static constexpr int ZRS = (ZN + 15) / 16 * 16;
   // shared memory, in doubles; SoA everywhere so a warp's LDS.64 is conflict-free
-  static constexpr int OFF_RAW = 0;                 // [3 slots][6 fields][RS] x,y,z,u,v,w (TMA)
-  static constexpr int OFF_ZR = OFF_RAW + 18 * RS;  // [3 slots][3 fields][ZRS] m, e, P (TMA)
+#ifndef HYDRO_MN8_TMA
+#define HYDRO_MN8_TMA 1
+#endif
+  static constexpr int NF = HYDRO_MN8_TMA ? 7 : 6;  // node fields: x,y,z,u,v,w[, 8/nodal mass]
+  static constexpr int OFF_RAW = 0;                 // [3 slots][NF fields][RS] (TMA)
+  static constexpr int OFF_ZR = OFF_RAW + 3 * NF * RS;  // [3 slots][3 fields][ZRS] m, e, P (TMA)
   static constexpr int OFF_XP = OFF_ZR + 9 * ZRS;   // [2 planes][3][RS] half-step positions
   static constexpr int OFF_G = OFF_XP + 6 * RS;     // [3 vectors][3][ZS] g_x, g_y, g_z
   static constexpr int OFF_UH = OFF_G + 9 * ZS;     // [3][ZS] u_half of node plane p
@@ -68,8 +72,8 @@ struct CTile {
 
 template <int TX, int TY, bool FUSED>
 __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
-    k_cycle(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st, int KZ,
-            int fold_finalize) {
+    k_cycle(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st, int tcols,
+            int ncols, int sched_kz, int fold_finalize) {
   using T = CTile<TX, TY>;
   // dynamic shared memory only (no static __shared__), so the window is 1024-byte aligned
   extern __shared__ __align__(1024) double sm[];
@@ -80,18 +84,49 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   constexpr int ZS = T::ZS, RS = T::RS, TXT = T::TXT, ZRS = T::ZRS, PX = T::PX;
 
   const int t = threadIdx.x;
-  const int i0 = blockIdx.x * TX, j0 = blockIdx.y * TY;
-  const int k0 = blockIdx.z * KZ;
-  const int k1 = min(k0 + KZ, d.n[2]);
   const int n0 = d.n[0], n1 = d.n[1], n2 = d.n[2];
   // lanes: zone/node (tx, ty) for tx < TXT; tx == TXT forms the box's last node column; the
   // rest (tx == PX-1 and the padding warp's tail) form the box's last node row
   const int tc = t;
   const int tx = t % PX, ty = t / PX;
   const bool active = t < T::NZT && tx < TXT;
+
+  // Work split (persistent, SM-count-sized grid; same scheme as kernel_zone.cu): the tile
+  // columns (TX x TY, all n2 zone planes) are linearised column-major into ncols * n2 units and
+  // CTA b takes [b W / G, (b+1) W / G), marched as one or two column segments.  sched_kz > 0:
+  // the chunked schedule (CTA b = column b / chunks, chunk b % chunks), for A/B measurement.
+  int64_t r0, r1;
+  if (sched_kz > 0) {
+    const int chunks = (n2 + sched_kz - 1) / sched_kz;
+    const int64_t col = blockIdx.x % ncols, ch = blockIdx.x / ncols;  // adjacent CTAs: same z
+    r0 = col * n2 + ch * sched_kz;
+    r1 = col * n2 + min((int)(ch + 1) * sched_kz, n2);
+  } else {
+    const int64_t W = (int64_t)ncols * n2;
+    r0 = W * blockIdx.x / gridDim.x;
+    r1 = W * (blockIdx.x + 1) / gridDim.x;
+  }
+  const bool halted = (st->halted | st->done) != 0u;
+  if (!halted && t == 0) {
+    if (smem_u32(sm) & 127u) __trap();  // TMA destinations must be 128-byte aligned
+    for (int s = 0; s < 3; ++s) mbar_init(&bar[s], 1);
+    for (int s = 3; s < 6; ++s) mbar_init(&bar[s], T::NTHR / 32);  // one arrival per warp
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  double dt2min = INFINITY;
+  uint32_t ubase = 0;  // TMA planes consumed in earlier segments (ring slot / phase continuity)
+  uint32_t pbase = 0;  // plane iterations run in earlier segments (phase-barrier parity)
+
+  for (int64_t r = r0; r < r1;) {
+  const int col = (int)(r / n2);
+  const int k0 = (int)(r - (int64_t)col * n2);
+  const int k1 = (int)min((int64_t)n2, r1 - (int64_t)col * n2);
+  r = (int64_t)col * n2 + k1;
+  const int i0 = (col % tcols) * TX, j0 = (col / tcols) * TY;
   const int li = i0 - 1 + tx, lj = j0 - 1 + ty;  // local zone / node index of this thread
 
-  if ((st->halted | st->done) != 0u) {  // no-op cycle: carry the state over to the next parity
+  if (halted) {  // no-op cycle: carry the state over to the next parity
     for (int p = k0; p <= k1; ++p) {
       if (!active || tx < 1 || ty < 1) continue;
       const bool wn = li <= n0 && lj <= n1 && (li < i0 + TX || li == n0) &&
@@ -106,7 +141,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
         d.en[z] = d.e[z];
       }
     }
-    return;
+    continue;
   }
 
   const double dt = st->dt;
@@ -118,22 +153,22 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   constexpr int NZF = FUSED ? 2 : 3;
   auto issue = [&](int q) {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    const int u = q - q0, s = u % 3;
-    double *dst = RAW + s * 6 * RS;
+    const uint32_t u = ubase + (uint32_t)(q - q0), s = u % 3;
+    double *dst = RAW + s * T::NF * RS;
     double *zdst = ZR + s * 3 * ZRS;
-    mbar_expect_tx(&bar[s], (6u * T::NN + (unsigned)NZF * T::ZN) * sizeof(double));
+    mbar_expect_tx(&bar[s], ((unsigned)T::NF * T::NN + (unsigned)NZF * T::ZN) * sizeof(double));
 #pragma unroll
-    for (int f = 0; f < 6; ++f) tma_load_3d(dst + f * RS, &maps.m[f], &bar[s], i0, j0, q + 1);
+    for (int f = 0; f < T::NF; ++f) tma_load_3d(dst + f * RS, &maps.m[f], &bar[s], i0, j0, q + 1);
 #pragma unroll
     for (int f = 0; f < NZF; ++f)  // FUSED: m, e; else 1/m (z[3]), e, P
       tma_load_3d(zdst + f * ZRS, &maps.z[(FUSED || f) ? f : 3], &bar[s], i0, j0, q + 1);
   };
   auto wait_plane = [&](int q) {
-    const int u = q - q0;
-    mbar_wait(&bar[u % 3], (uint32_t)((u / 3) & 1));
+    const uint32_t u = ubase + (uint32_t)(q - q0);
+    mbar_wait(&bar[u % 3], (u / 3) & 1u);
   };
-  auto raw = [&](int q) { return RAW + ((q - q0) % 3) * 6 * RS; };
-  auto zraw = [&](int q) { return ZR + ((q - q0) % 3) * 3 * ZRS; };
+  auto raw = [&](int q) { return RAW + ((ubase + (uint32_t)(q - q0)) % 3) * T::NF * RS; };
+  auto zraw = [&](int q) { return ZR + ((ubase + (uint32_t)(q - q0)) % 3) * 3 * ZRS; };
   // X stage: half-step positions of node plane q into XP slot q&1.  Thread t forms its own
   // node (tx, ty) -- returned in registers -- and the box's last column / row are shared out.
   const int nidx = t;  // this thread's node in the node box (pitch PX)
@@ -167,15 +202,10 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   };
 
   if (t == 0) {
-    if (smem_u32(sm) & 127u) __trap();  // TMA destinations must be 128-byte aligned
-    for (int s = 0; s < 3; ++s) mbar_init(&bar[s], 1);
-    for (int s = 3; s < 6; ++s) mbar_init(&bar[s], T::NTHR / 32);  // one arrival per warp
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     issue(q0);
     issue(q0 + 1);
     if (q0 + 2 <= k1 + 1) issue(q0 + 2);
   }
-  __syncthreads();
 
   // Values one plane hands to the next.  Two sets alternate (the loop body runs twice per trip
   // with the roles swapped), so nothing is copied between iterations: iteration p reads plane
@@ -192,7 +222,6 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   };
   struct XP3 { double x, y, z; };  // own node's half-step position
   Carry S0 = {}, S1 = {};
-  double dt2min = INFINITY;
 
   // Per-thread constants, kept in few registers (32-bit indices: a domain's storage is below
   // 2^31 elements, checked at create) so the compiler does not rematerialise them per plane.
@@ -242,7 +271,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     __syncwarp();
     if ((t & 31) == 0) mbar_arrive(&bar[b]);
   };
-  auto await = [&](int b, int p) { mbar_wait(&bar[b], (uint32_t)((p - q0) & 1)); };
+  auto await = [&](int b, int p) { mbar_wait(&bar[b], (pbase + (uint32_t)(p - q0)) & 1u); };
   auto energy2 = [&](int zp, const Carry &c) {  // E2 of zone plane zp from its carry set
     if (fl & F_OWN) {
       const double Wk = 0.125 * c.P * ((PSX[t + 1] + PSY[t + PX]) + c.part);
@@ -251,8 +280,9 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   };
 
   auto body = [&](const int p, Carry &pv, Carry &cu, XP3 &xa, const XP3 &xb) {
-    // 8 / nodal mass of this thread's node on plane p (read early: its latency hides under Z)
-    const double rinv_n = ((fl & F_NODE) && p >= k0) ? __ldg(d.mn8 + (p + 1) * nsxy + nrow) : 0.0;
+    // (HYDRO_MN8_TMA=0) 8 / nodal mass from global memory, read early so its latency hides
+    const double rinv_g = (!HYDRO_MN8_TMA && (fl & F_NODE) && p >= k0)
+                              ? __ldg(d.mn8 + (p + 1) * nsxy + nrow) : 0.0;
     // ---------------------------------------------------------------- phase 1: E2(p-2), Z(p)
     if (FUSED && p >= k0 + 2) energy2(p - 2, cu);  // cu still holds zone plane p-2
     const bool exists = (fl & F_ZEX) && p >= gz_lo && p < gz_hi;
@@ -396,7 +426,8 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
         const double Fx = pv.Sx + Cx + ((a0 + b0) + fma(gzw, cx0, c0));
         const double Fy = pv.Sy + Cy + ((a1 + b1) + fma(gzw, cy0, c1));
         const double Fz = pv.Sz + Cz + ((a2_ + b2) + fma(gzw, cz0, c2_));
-        const double rinv = rinv_n;  // 8 / nodal mass (constant, d.mn8)
+        const double rinv =  // 8 / nodal mass (constant d.mn8)
+            HYDRO_MN8_TMA ? Ra[6 * RS + nidx] : rinv_g;
         const bool wall_z = p == wz_lo || p == wz_hi;
         const double axc = (fl & F_WX) ? 0.0 : Fx * rinv;
         const double ayc = (fl & F_WY) ? 0.0 : Fy * rinv;
@@ -474,6 +505,10 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     if (p + 1 > k1) break;
     body(p + 1, S1, S0, XB, XA);
   }
+  ubase += (uint32_t)(k1 + 2 - q0);  // node planes q0 .. k1+1 went through the TMA ring
+  pbase += (uint32_t)(k1 + 1 - q0);  // iterations p = q0 .. k1 completed each phase barrier
+  __syncthreads();                   // the next segment reuses the rings
+  }
   if (FUSED) block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);
   if (fold_finalize)  // single-domain, single-rank cycle: S9 here instead of a separate launch
     finalize_if_last_block(st, ph, reinterpret_cast<unsigned int *>(sm + T::OFF_RED));
@@ -481,7 +516,8 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
 
 constexpr int CTX = 32, CTY = 12;
 
-// z-chunk length: minimise (waves of blocks) x (planes per block incl. the 2 warm-up planes).
+// z-chunk length of the chunked schedule: minimise (waves of CTAs) x (planes per CTA incl. the
+// 2 warm-up planes).
 int choose_kz(int tiles, int n2, int sms) {
   int best = n2, best_cost = 1 << 30;
   for (int kz = 4; kz <= n2; ++kz) {
@@ -509,11 +545,21 @@ void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st
                          (int)T::BYTES);
   }
   const int tx = (d.n[0] + CTX - 1) / CTX, ty = (d.n[1] + CTY - 1) / CTY;
+  // Default: the chunked schedule (CTAs adjacent in x, y at the same z-chunk, so the tile rings
+  // that neighbouring CTAs both read are L2 hits; measured faster here than the persistent
+  // linearised split, which spreads concurrent CTAs over z: 94 vs 110 us at 128^3).
+  // HYDRO_KZ_NODE / HYDRO_KZ_FUSED = k: chunks of k planes; = -1: the persistent split.
   static const int kz_env = getenv(FUSED ? "HYDRO_KZ_FUSED" : "HYDRO_KZ_NODE")
                                 ? atoi(getenv(FUSED ? "HYDRO_KZ_FUSED" : "HYDRO_KZ_NODE")) : 0;
-  const int KZ = kz_env > 0 ? std::min(kz_env, d.n[2]) : choose_kz(tx * ty, d.n[2], sms);
-  dim3 grid(tx, ty, (d.n[2] + KZ - 1) / KZ);
-  k_cycle<CTX, CTY, FUSED><<<grid, T::NTHR, T::BYTES, s>>>(maps, d, ph, st, KZ, fold);
+  const int ncols = tx * ty;
+  int G, kz = 0;
+  if (kz_env >= 0) {
+    kz = kz_env > 0 ? std::min(kz_env, d.n[2]) : choose_kz(ncols, d.n[2], sms);
+    G = ncols * ((d.n[2] + kz - 1) / kz);
+  } else {
+    G = (int)std::min<int64_t>(sms, (int64_t)ncols * d.n[2]);
+  }
+  k_cycle<CTX, CTY, FUSED><<<G, T::NTHR, T::BYTES, s>>>(maps, d, ph, st, tx, ncols, kz, fold);
 }
 
 }  // namespace

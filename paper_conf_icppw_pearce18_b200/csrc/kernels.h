@@ -36,10 +36,11 @@ void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, cudaStrea
 void launch_node_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 void launch_energy_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 
-// TMA descriptors of one domain and parity: the six node-state arrays (x,y,z,u,v,w) and the
+// TMA descriptors of one domain and parity: the six node-state arrays (x,y,z,u,v,w), the
+// constant nodal 8/mass array and the
 // zone arrays m, e, P (box = the kernel's zone tile).
 struct alignas(64) NodeMaps {
-  CUtensorMap m[6];
+  CUtensorMap m[7];  // x, y, z, u, v, w, 8/nodal mass
   CUtensorMap z[4];  // m, e, P, 1/m
 };
 

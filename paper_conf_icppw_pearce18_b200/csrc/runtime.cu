@@ -158,15 +158,15 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
     encode = (PFN_cuTensorMapEncodeTiled_v12000)fn;
   }
   for (int par = 0; par < 2; ++par) {
-    const double *arr[6] = {D.view[par].x, D.view[par].y, D.view[par].z,
-                            D.view[par].u, D.view[par].v, D.view[par].w};
+    const double *arr[7] = {D.view[par].x, D.view[par].y, D.view[par].z,
+                            D.view[par].u, D.view[par].v, D.view[par].w, D.view[par].mn8};
     const double *zarr[4] = {D.view[par].m, D.view[par].e, D.view[par].P, D.view[par].mi};
     for (int kind = 0; kind < 2; ++kind) {
       if (kind == 0 && fused_box_y() != node_box_y())
         return set_err(h, HYDRO_EINVAL, "fused and node kernels must share a TMA box");
       NodeMaps &M = kind ? D.zmaps[par] : D.maps[par];
-      for (int f = 0; f < 10; ++f) {
-        const bool zf = f >= 6;
+      for (int f = 0; f < 11; ++f) {
+        const bool zf = f >= 6 && f < 10;
         const int64_t sx = zf ? zsx : nsx, sy = zf ? (n1 + 2) : (n1 + 3);
         const int64_t sz = zf ? (n2 + 2) : (n2 + 3), sxy = zf ? zsxy : nsxy;
         cuuint64_t dims[3] = {(cuuint64_t)sx, (cuuint64_t)sy, (cuuint64_t)sz};
@@ -182,9 +182,9 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
         }
         box[2] = 1;
         cuuint32_t es[3] = {1, 1, 1};
-        CUtensorMap *dst = zf ? &M.z[f - 6] : &M.m[f];
+        CUtensorMap *dst = zf ? &M.z[f - 6] : &M.m[f == 10 ? 6 : f];
         CUresult r = encode(dst, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3,
-                            const_cast<double *>(zf ? zarr[f - 6] : arr[f]), dims, strides, box,
+                            const_cast<double *>(zf ? zarr[f - 6] : arr[f == 10 ? 6 : f]), dims, strides, box,
                             es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
                             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
         if (r != CUDA_SUCCESS) return set_err(h, HYDRO_ECUDA, "cuTensorMapEncodeTiled failed");

@@ -16,7 +16,8 @@ from typing import Dict, Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libhydro_b200.so")
+# HYDRO_LIB: an alternative build of the same library (A/B measurements of kernel variants)
+LIB_PATH = os.environ.get("HYDRO_LIB") or os.path.join(_HERE, "libhydro_b200.so")
 
 NODE_FIELDS = ("x", "y", "z", "u", "v", "w")
 ZONE_FIELDS = ("rho", "e", "p", "q", "c", "vol", "mass")
