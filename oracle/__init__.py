@@ -50,6 +50,8 @@ def lib() -> C.CDLL:
         L.orc_zone_geometry.restype = None
         L.orc_zone_state.argtypes = [C.c_void_p, C.c_void_p] + [C.c_double] * 8 + [C.c_void_p]
         L.orc_zone_state.restype = None
+        L.orc_zone_hourglass.argtypes = [C.c_void_p] * 3 + [C.c_double] * 4 + [C.c_void_p]
+        L.orc_zone_hourglass.restype = None
         _lib = L
     return _lib
 
@@ -69,6 +71,7 @@ class _Config(C.Structure):
         ("init_kind", C.c_int32),
         ("rho0", C.c_double), ("e0", C.c_double), ("sedov_energy", C.c_double),
         ("user", C.POINTER(C.c_double) * 8),
+        ("hg_coef", C.c_double),
     ]
 
 
@@ -105,6 +108,7 @@ class OracleConfig:
     e0: float = 0.0
     sedov_energy: float = 0.851072 / 8.0   # reading R10: octant share, R(t=1)=1 for gamma=1.4
     user: Optional[Dict[str, np.ndarray]] = None
+    hg_coef: float = 0.0                  # reading R17 / SURVEY §8f f1: hourglass kappa, 0 = off
 
 
 class OracleError(RuntimeError):
@@ -132,7 +136,7 @@ class Oracle:
                 self._keep.append(arr)
                 c.cuts[a] = arr.ctypes.data_as(C.POINTER(C.c_int64))
         for k in ("gamma", "q_lin", "q_quad", "cfl", "c_vol", "dt_growth", "dt_max", "dt_init",
-                  "t_stop", "dt_first", "t0", "rho0", "e0", "sedov_energy"):
+                  "t_stop", "dt_first", "t0", "rho0", "e0", "sedov_energy", "hg_coef"):
             setattr(c, k, float(getattr(cfg, k)))
         c.reflect_mask = int(cfg.reflect_mask)
         c.init_kind = INIT[cfg.init]
@@ -214,6 +218,17 @@ def zone_state(X, U, m, e, hh, gamma=1.4, q_lin=0.5, q_quad=2.0, cfl=0.3, c_vol=
                          float(gamma), float(q_lin), float(q_quad), float(cfl), float(c_vol),
                          out.ctypes.data)
     return dict(zip(("rho", "ep", "p", "c", "q", "P", "dtz", "V"), out.tolist()))
+
+
+def zone_hourglass(X, U, B, V, rho, c, kappa) -> np.ndarray:
+    """f1 / reading R17: Flanagan-Belytschko hourglass corner forces of one zone (8, 3)."""
+    X = np.ascontiguousarray(X, dtype=np.float64).reshape(8, 3)
+    U = np.ascontiguousarray(U, dtype=np.float64).reshape(8, 3)
+    B = np.ascontiguousarray(B, dtype=np.float64).reshape(8, 3)
+    F = np.zeros((8, 3))
+    lib().orc_zone_hourglass(X.ctypes.data, U.ctypes.data, B.ctypes.data, float(V), float(rho),
+                             float(c), float(kappa), F.ctypes.data)
+    return F
 
 
 def run(cfg: OracleConfig, ncycles: int, names: Sequence[str] = ALL_FIELDS):

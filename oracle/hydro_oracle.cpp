@@ -93,6 +93,7 @@ void geometry(const double X[8][3], double B[8][3], double *V, double *L) {
 
 struct Params {
   double gamma, gm1, ggm1, q_lin, q_quad, cfl, c_vol;
+  double hg;  // hourglass coefficient kappa (reading R17; 0 = off)
 };
 
 struct ZoneOut {
@@ -144,6 +145,79 @@ void zone_state(const double X[8][3], const double U[8][3], double m, double e, 
   o->D = D;
 }
 
+// S5 addition, SURVEY §8f row f1 / reading R17: viscous hourglass control in
+// the Flanagan-Belytschko form, added to the corner forces f_l = P B_l (so it is still a corner
+// force: momentum and, through the compatible S8 update, total energy stay conserved).
+//   base vectors on the reference cube, corner l = a+2b+4c, xi = 2a-1, eta = 2b-1, zeta = 2c-1:
+//     h1 = eta*zeta, h2 = zeta*xi, h3 = xi*eta, h4 = xi*eta*zeta;
+//   M_dk = sum_l B_ld X_lk  (= V delta_dk when B is the exact gradient of V: affine hexes),
+//   H_ak = sum_l h_al X_lk,  C = H M^-1,
+//   gamma_al = h_al - sum_d C_ad B_ld   (sum_l gamma_al = 0 and sum_l gamma_al X_lk = 0 exactly
+//                                        in real arithmetic: linear velocity fields are immune),
+//   g_ad = sum_l gamma_al U_ld,
+//   f_hg_ld = -kappa rho c V^(2/3) sum_a gamma_al g_ad.
+// X: half-step positions, U: u^n, B/V/rho/c: the zone's S2-S3 values (same as for P).
+void hourglass(const double X[8][3], const double U[8][3], const double B[8][3], double V,
+               double rho, double c, double kappa, double F[8][3]) {
+  double h[4][8];
+  for (int l = 0; l < 8; ++l) {
+    const double xi = 2.0 * (l & 1) - 1.0, eta = 2.0 * ((l >> 1) & 1) - 1.0,
+                 zeta = 2.0 * ((l >> 2) & 1) - 1.0;
+    h[0][l] = eta * zeta;
+    h[1][l] = zeta * xi;
+    h[2][l] = xi * eta;
+    h[3][l] = (xi * eta) * zeta;
+  }
+  double M[3][3], H[4][3];
+  for (int d = 0; d < 3; ++d)
+    for (int k = 0; k < 3; ++k) {
+      double sum = 0.0;
+      for (int l = 0; l < 8; ++l) sum = (l == 0) ? B[l][d] * X[l][k] : sum + B[l][d] * X[l][k];
+      M[d][k] = sum;
+    }
+  for (int a = 0; a < 4; ++a)
+    for (int k = 0; k < 3; ++k) {
+      double sum = 0.0;
+      for (int l = 0; l < 8; ++l) sum = (l == 0) ? h[a][l] * X[l][k] : sum + h[a][l] * X[l][k];
+      H[a][k] = sum;
+    }
+  // M^-1 by the adjugate: Minv[k][d] = cof(M)[d][k] / det M
+  double cof[3][3];
+  for (int r = 0; r < 3; ++r)
+    for (int q = 0; q < 3; ++q) {
+      const int r1 = (r + 1) % 3, r2 = (r + 2) % 3, q1 = (q + 1) % 3, q2 = (q + 2) % 3;
+      cof[r][q] = M[r1][q1] * M[r2][q2] - M[r1][q2] * M[r2][q1];
+    }
+  const double det = (M[0][0] * cof[0][0] + M[0][1] * cof[0][1]) + M[0][2] * cof[0][2];
+  double Minv[3][3];
+  for (int k = 0; k < 3; ++k)
+    for (int d = 0; d < 3; ++d) Minv[k][d] = cof[d][k] / det;
+  double C[4][3];
+  for (int a = 0; a < 4; ++a)
+    for (int d = 0; d < 3; ++d)
+      C[a][d] = (H[a][0] * Minv[0][d] + H[a][1] * Minv[1][d]) + H[a][2] * Minv[2][d];
+  double gam[4][8];
+  for (int a = 0; a < 4; ++a)
+    for (int l = 0; l < 8; ++l)
+      gam[a][l] = h[a][l] - ((C[a][0] * B[l][0] + C[a][1] * B[l][1]) + C[a][2] * B[l][2]);
+  double g[4][3];
+  for (int a = 0; a < 4; ++a)
+    for (int d = 0; d < 3; ++d) {
+      double sum = 0.0;
+      for (int l = 0; l < 8; ++l)
+        sum = (l == 0) ? gam[a][l] * U[l][d] : sum + gam[a][l] * U[l][d];
+      g[a][d] = sum;
+    }
+  const double v13 = std::cbrt(V);
+  const double coef = -(((kappa * rho) * c) * (v13 * v13));
+  for (int l = 0; l < 8; ++l)
+    for (int d = 0; d < 3; ++d) {
+      double sum = 0.0;
+      for (int a = 0; a < 4; ++a) sum = (a == 0) ? gam[a][l] * g[a][d] : sum + gam[a][l] * g[a][d];
+      F[l][d] = coef * sum;
+    }
+}
+
 // ----------------------------------------------------------------------------------------
 // Domains.  Owned zones [lo, lo+n) per axis (global).  Local zone index i in [-1, n] and node
 // index i in [-1, n+1]; storage offset +1.  Only entries that exist in the global mesh are
@@ -152,6 +226,7 @@ struct Domain {
   int64_t lo[3], n[3], zs[3], ns[3];
   std::vector<double> x[3], u[3], xn[3], un[3], xp[3], uh[3];
   std::vector<double> m, e, en, P, B;  // B: 24 per zone
+  std::vector<double> HG;              // hourglass corner forces, 24 per zone (kappa > 0 only)
   std::vector<uint8_t> zex, nex;       // exists in the global mesh
 
   int64_t zid(int64_t i, int64_t j, int64_t k) const {
@@ -234,6 +309,7 @@ void init_domain(orc_ctx *h, Domain &D) {
   D.en.assign(tot_z, 0.0);
   D.P.assign(tot_z, 0.0);
   D.B.assign(tot_z * 24, 0.0);
+  if (h->pr.hg > 0.0) D.HG.assign(tot_z * 24, 0.0);
   D.zex.assign(tot_z, 0);
   D.nex.assign(tot_n, 0);
   for (int64_t k = -1; k <= D.n[2] + 1; ++k)
@@ -356,6 +432,11 @@ void cycle(orc_ctx *h) {
           zone_state(X, U, D.m[id], D.e[id], hh, h->pr, B, &o);
           std::memcpy(&D.B[id * 24], B, sizeof(B));
           D.P[id] = o.P;  // S5 f_l = P*B_l is formed where it is used (same bits)
+          if (h->pr.hg > 0.0) {  // f1: f_l = P*B_l + f_hg_l
+            double Fh[8][3];
+            hourglass(X, U, B, o.V, o.rho, o.c, h->pr.hg, Fh);
+            std::memcpy(&D.HG[id * 24], Fh, sizeof(Fh));
+          }
           const bool owned = i >= 0 && i < D.n[0] && j >= 0 && j < D.n[1] && k >= 0 &&
                              k < D.n[2];
           if (!owned) continue;
@@ -378,7 +459,10 @@ void cycle(orc_ctx *h) {
             if (!D.zex[zid]) continue;
             const double *Bz = &D.B[zid * 24 + (7 - lp) * 3];
             const double P = D.P[zid];
-            for (int d = 0; d < 3; ++d) F[d] = first ? P * Bz[d] : F[d] + P * Bz[d];
+            double f[3] = {P * Bz[0], P * Bz[1], P * Bz[2]};
+            if (h->pr.hg > 0.0)
+              for (int d = 0; d < 3; ++d) f[d] = f[d] + D.HG[zid * 24 + (7 - lp) * 3 + d];
+            for (int d = 0; d < 3; ++d) F[d] = first ? f[d] : F[d] + f[d];
             msum = first ? D.m[zid] : msum + D.m[zid];
             first = false;
           }
@@ -411,7 +495,9 @@ void cycle(orc_ctx *h) {
           for (int l = 0; l < 8; ++l) {
             const int64_t nid = D.nid(i + (l & 1), j + ((l >> 1) & 1), k + ((l >> 2) & 1));
             const double *Bl = &D.B[id * 24 + l * 3];
-            const double f[3] = {P * Bl[0], P * Bl[1], P * Bl[2]};
+            double f[3] = {P * Bl[0], P * Bl[1], P * Bl[2]};
+            if (h->pr.hg > 0.0)
+              for (int d = 0; d < 3; ++d) f[d] = f[d] + D.HG[id * 24 + l * 3 + d];
             const double uh[3] = {D.uh[0][nid], D.uh[1][nid], D.uh[2][nid]};
             const double t = dot3(f, uh);
             W = (l == 0) ? t : W + t;
@@ -452,7 +538,7 @@ bool valid_config(const orc_config *c) {
     }
   }
   if (!(c->gamma > 1.0) || c->q_lin < 0.0 || c->q_quad < 0.0 || !(c->cfl > 0.0) ||
-      !(c->c_vol > 0.0) || !(c->dt_growth > 0.0) || !(c->dt_max > 0.0))
+      !(c->c_vol > 0.0) || !(c->dt_growth > 0.0) || !(c->dt_max > 0.0) || !(c->hg_coef >= 0.0))
     return false;
   if (c->init_kind != ORC_INIT_SEDOV) {
     for (int f = 0; f < 8; ++f)
@@ -467,6 +553,11 @@ extern "C" {
 
 const char *orc_last_error(void) { return g_err.c_str(); }
 
+void orc_zone_hourglass(const double X[8][3], const double U[8][3], const double B[8][3],
+                        double V, double rho, double c, double kappa, double F[8][3]) {
+  hourglass(X, U, B, V, rho, c, kappa, F);
+}
+
 void orc_zone_geometry(const double X[8][3], double B[8][3], double *V, double *L) {
   geometry(X, B, V, L);
 }
@@ -474,7 +565,7 @@ void orc_zone_geometry(const double X[8][3], double B[8][3], double *V, double *
 void orc_zone_state(const double X[8][3], const double U[8][3], double m, double e, double hh,
                     double gamma, double q_lin, double q_quad, double cfl, double c_vol,
                     double out[8]) {
-  Params pr{gamma, gamma - 1.0, gamma * (gamma - 1.0), q_lin, q_quad, cfl, c_vol};
+  Params pr{gamma, gamma - 1.0, gamma * (gamma - 1.0), q_lin, q_quad, cfl, c_vol, 0.0};
   double B[8][3];
   ZoneOut o;
   zone_state(X, U, m, e, hh, pr, B, &o);
@@ -522,7 +613,7 @@ int orc_create(const orc_config *cfg, orc_ctx **out) {
   h->ndy = cfg->ndom[1];
   h->ndz = cfg->ndom[2];
   h->pr = Params{cfg->gamma, cfg->gamma - 1.0, cfg->gamma * (cfg->gamma - 1.0), cfg->q_lin,
-                 cfg->q_quad, cfg->cfl, cfg->c_vol};
+                 cfg->q_quad, cfg->cfl, cfg->c_vol, cfg->hg_coef};
   h->dom.resize((size_t)h->ndx * h->ndy * h->ndz);
   for (int c = 0; c < h->ndz; ++c)
     for (int b = 0; b < h->ndy; ++b)

@@ -49,6 +49,7 @@ typedef struct {
   /* USER / USER_MASS: global arrays, x fastest.  [0..5] = x,y,z,u,v,w on (n+1)^3 nodes;
      [6] = rho (USER) or zone mass (USER_MASS) on n^3 zones; [7] = e on zones. */
   const double *user[8];
+  double hg_coef;               /* viscous hourglass coefficient kappa >= 0 (reading R17; 0 = off) */
 } orc_config;
 
 typedef struct {
@@ -86,6 +87,11 @@ void orc_zone_geometry(const double X[8][3], double B[8][3], double *V, double *
 void orc_zone_state(const double X[8][3], const double U[8][3], double m, double e, double hh,
                     double gamma, double q_lin, double q_quad, double cfl, double c_vol,
                     double out[8] /* rho, e_p, p, c, q, P, dt_z, V */);
+
+/* f1 (reading R17): Flanagan-Belytschko viscous hourglass corner forces of one zone, from the
+   half-step positions X, velocities U, corner vectors B, V, rho, c and kappa (hydro_oracle.cpp). */
+void orc_zone_hourglass(const double X[8][3], const double U[8][3], const double B[8][3],
+                        double V, double rho, double c, double kappa, double F[8][3]);
 
 #ifdef __cplusplus
 }
