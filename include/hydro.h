@@ -35,7 +35,7 @@
 extern "C" {
 #endif
 
-#define HYDRO_ABI_VERSION 1
+#define HYDRO_ABI_VERSION 2
 
 typedef struct hydro_ctx hydro_ctx; /* opaque; owned by the library */
 
@@ -101,6 +101,11 @@ typedef struct {
   const void *comm_id;          /* nranks > 1: 128-byte id from hydro_comm_unique_id() on rank 0,
                                    broadcast by the caller (e.g. torch.distributed) */
   uint64_t flags;               /* HYDRO_FLAG_* */
+  double hg_coef;               /* viscous hourglass coefficient kappa >= 0 (SURVEY §8f row f1,
+                                   reading R17): f_l += -kappa rho c V^(2/3) sum_a gamma_al g_a
+                                   (Flanagan-Belytschko).  0 = off (the default,
+                                   north_star's phase list).  kappa > 0 runs the split kernels
+                                   (corner-force planes in HBM), whatever the path flags say. */
 } hydro_config;
 
 typedef struct {

@@ -47,6 +47,7 @@ struct Phys {
   double dt_growth, dt_max, t_stop;
   uint32_t reflect_mask;
   uint32_t pad_;
+  double hg;  // hourglass kappa (split path only; 0 = off)
 };
 
 // Device-resident scalar state of a run (one per rank).  Kernels read t, dt from here so a

@@ -173,11 +173,21 @@ __global__ void k_zone_split(DomView d, Phys ph, DevState *st) {
     const int64_t id = d.zid(i, j, k);
     const ZoneEos r = zone_eos(V, A2, DV, d.m[id], d.e[id], hh, ph);
     d.P[id] = r.P;
+    // S5 corner forces f_l = P B_l (+ the f1 hourglass force), 24 planes for K2 and K3
+    double Fx[8], Fy[8], Fz[8];
 #pragma unroll
     for (int l = 0; l < 8; ++l) {
-      d.B[(3 * l + 0) * d.nzone + id] = Bx[l];
-      d.B[(3 * l + 1) * d.nzone + id] = By[l];
-      d.B[(3 * l + 2) * d.nzone + id] = Bz[l];
+      Fx[l] = r.P * Bx[l];
+      Fy[l] = r.P * By[l];
+      Fz[l] = r.P * Bz[l];
+    }
+    if (ph.hg > 0.0)
+      hourglass_add(X, Y, Z, U, Vv, W, Bx, By, Bz, V, r.rho, r.c, ph.hg, Fx, Fy, Fz);
+#pragma unroll
+    for (int l = 0; l < 8; ++l) {
+      d.B[(3 * l + 0) * d.nzone + id] = Fx[l];
+      d.B[(3 * l + 1) * d.nzone + id] = Fy[l];
+      d.B[(3 * l + 2) * d.nzone + id] = Fz[l];
     }
     const bool owned = i >= 0 && j >= 0 && k >= 0 && i < d.n[0] && j < d.n[1] && k < d.n[2];
     if (owned) {
@@ -189,7 +199,7 @@ __global__ void k_zone_split(DomView d, Phys ph, DevState *st) {
   block_min_dt(dtz, &st->dtz_acc);
 }
 
-// K2: S5 + S7 for owned nodes: gather f = P*B from the existing zones around the node,
+// K2: S5 + S7 for owned nodes: gather the corner forces f from the existing zones around the node,
 // acceleration, reflecting walls, velocity and position update.
 __global__ void k_node_split(DomView d, Phys ph, DevState *st) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
@@ -210,10 +220,9 @@ __global__ void k_node_split(DomView d, Phys ph, DevState *st) {
     if (!exists_zone(d, zi, zj, zk)) continue;
     const int64_t z = d.zid(zi, zj, zk);
     const int l = 7 - lp;
-    const double P = d.P[z];
-    Fx += P * d.B[(3 * l + 0) * d.nzone + z];
-    Fy += P * d.B[(3 * l + 1) * d.nzone + z];
-    Fz += P * d.B[(3 * l + 2) * d.nzone + z];
+    Fx += d.B[(3 * l + 0) * d.nzone + z];
+    Fy += d.B[(3 * l + 1) * d.nzone + z];
+    Fz += d.B[(3 * l + 2) * d.nzone + z];
     ms += d.m[z];
   }
   const double rinv = 1.0 / (0.125 * ms);
@@ -234,7 +243,7 @@ __global__ void k_node_split(DomView d, Phys ph, DevState *st) {
   d.zn[id] = d.z[id] + dt * wh;
 }
 
-// K3: S8 for owned zones: W = sum_l (P B_l).u_half_l, e' = e - dt W / m.
+// K3: S8 for owned zones: W = sum_l f_l.u_half_l, e' = e - dt W / m.
 __global__ void k_energy_split(DomView d, Phys ph, DevState *st) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   const int j = blockIdx.y * blockDim.y + threadIdx.y;
@@ -246,7 +255,6 @@ __global__ void k_energy_split(DomView d, Phys ph, DevState *st) {
     return;
   }
   const double dt = st->dt;
-  const double P = d.P[id];
   double Wk = 0.0;
 #pragma unroll
   for (int l = 0; l < 8; ++l) {
@@ -254,8 +262,8 @@ __global__ void k_energy_split(DomView d, Phys ph, DevState *st) {
     const double uh = (d.u[n] + d.un[n]) * 0.5;
     const double vh = (d.v[n] + d.vn[n]) * 0.5;
     const double wh = (d.w[n] + d.wn[n]) * 0.5;
-    Wk += (P * d.B[(3 * l + 0) * d.nzone + id]) * uh + (P * d.B[(3 * l + 1) * d.nzone + id]) * vh +
-          (P * d.B[(3 * l + 2) * d.nzone + id]) * wh;
+    Wk += d.B[(3 * l + 0) * d.nzone + id] * uh + d.B[(3 * l + 1) * d.nzone + id] * vh +
+          d.B[(3 * l + 2) * d.nzone + id] * wh;
   }
   d.en[id] = d.e[id] - dt * Wk / d.m[id];
 }

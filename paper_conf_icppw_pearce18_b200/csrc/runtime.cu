@@ -379,7 +379,7 @@ bool valid_phys(const hydro_config *c) {
   return c->gamma > 1.0 && c->q_lin >= 0.0 && c->q_quad >= 0.0 && c->cfl > 0.0 &&
          c->c_vol > 0.0 && c->dt_growth > 0.0 && c->dt_max > 0.0 &&
          std::isfinite(c->origin[0]) && c->extent[0] > 0.0 && c->extent[1] > 0.0 &&
-         c->extent[2] > 0.0;
+         c->extent[2] > 0.0 && c->hg_coef >= 0.0 && std::isfinite(c->hg_coef);
 }
 
 }  // namespace
@@ -467,7 +467,9 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
   h->ph.dt_max = cfg->dt_max;
   h->ph.t_stop = cfg->t_stop;
   h->ph.reflect_mask = cfg->reflect_mask;
-  h->split = (cfg->flags & HYDRO_FLAG_SPLIT) != 0;
+  h->ph.hg = cfg->hg_coef;
+  // hourglass control (f1) needs per-corner forces, which only the split kernels carry
+  h->split = (cfg->flags & HYDRO_FLAG_SPLIT) != 0 || cfg->hg_coef > 0.0;
   h->one_kernel = !h->split && (cfg->flags & HYDRO_FLAG_ONE_KERNEL) != 0;
   h->use_graph = (cfg->flags & HYDRO_FLAG_NO_GRAPH) == 0;
   h->device = cfg->device;

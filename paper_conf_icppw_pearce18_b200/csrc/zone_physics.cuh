@@ -57,6 +57,89 @@ __device__ __forceinline__ void hex_geometry(const double X[8], const double Y[8
   A2max = a2;
 }
 
+// f1 (reading R17): viscous hourglass corner forces, Flanagan-Belytschko form,
+// added to P B_l.  Hourglass base vectors h_a,l in {-1, +1} (a = 0..3: eta zeta, zeta xi, xi eta,
+// xi eta zeta with xi = +-1 by corner bit a, ...).  The projection uses C = H M^-1 with
+// M_dk = sum_l B_l,d X_l,k and H_ak = sum_l h_a,l X_l,k, so gamma_a = h_a - C_a . B is orthogonal
+// to every linear field on any hex; g_a = sum_l gamma_a,l u_l (u^n); the corner force is
+// f_l = -kappa rho c V^(2/3) sum_a gamma_a,l g_a.  Adds into F (x, y, z per corner).
+__device__ __forceinline__ double hg_sign(int a, int l) {
+  const double xi = (l & 1) ? 1.0 : -1.0, eta = (l & 2) ? 1.0 : -1.0, zeta = (l & 4) ? 1.0 : -1.0;
+  return a == 0 ? eta * zeta : a == 1 ? zeta * xi : a == 2 ? xi * eta : xi * eta * zeta;
+}
+__device__ __forceinline__ void hourglass_add(const double X[8], const double Y[8],
+                                              const double Z[8], const double U[8],
+                                              const double Vv[8], const double W[8],
+                                              const double Bx[8], const double By[8],
+                                              const double Bz[8], double V, double rho, double c,
+                                              double kappa, double Fx[8], double Fy[8],
+                                              double Fz[8]) {
+  const double *P3[3] = {X, Y, Z};
+  const double *B3[3] = {Bx, By, Bz};
+  double M[3][3], H[4][3];
+#pragma unroll
+  for (int d = 0; d < 3; ++d)
+#pragma unroll
+    for (int k = 0; k < 3; ++k) {
+      double s = 0.0;
+#pragma unroll
+      for (int l = 0; l < 8; ++l) s = fma(B3[d][l], P3[k][l], s);
+      M[d][k] = s;
+    }
+#pragma unroll
+  for (int a = 0; a < 4; ++a)
+#pragma unroll
+    for (int k = 0; k < 3; ++k) {
+      double s = 0.0;
+#pragma unroll
+      for (int l = 0; l < 8; ++l) s += hg_sign(a, l) * P3[k][l];
+      H[a][k] = s;
+    }
+  // adjugate inverse: (M^-1)_kd = adj(M)_kd / det = cof(M)_dk / det
+  double cf[3][3];
+#pragma unroll
+  for (int r = 0; r < 3; ++r)
+#pragma unroll
+    for (int q = 0; q < 3; ++q)
+      cf[r][q] = M[(r + 1) % 3][(q + 1) % 3] * M[(r + 2) % 3][(q + 2) % 3] -
+                 M[(r + 1) % 3][(q + 2) % 3] * M[(r + 2) % 3][(q + 1) % 3];
+  const double idet = 1.0 / (M[0][0] * cf[0][0] + M[0][1] * cf[0][1] + M[0][2] * cf[0][2]);
+  double C[4][3];
+#pragma unroll
+  for (int a = 0; a < 4; ++a)
+#pragma unroll
+    for (int d = 0; d < 3; ++d)
+      C[a][d] = (H[a][0] * cf[d][0] + H[a][1] * cf[d][1] + H[a][2] * cf[d][2]) * idet;
+  double gam[4][8], g[4][3];
+#pragma unroll
+  for (int a = 0; a < 4; ++a) {
+    double gx = 0.0, gy = 0.0, gz = 0.0;
+#pragma unroll
+    for (int l = 0; l < 8; ++l) {
+      gam[a][l] = hg_sign(a, l) - (C[a][0] * Bx[l] + C[a][1] * By[l] + C[a][2] * Bz[l]);
+      gx = fma(gam[a][l], U[l], gx);
+      gy = fma(gam[a][l], Vv[l], gy);
+      gz = fma(gam[a][l], W[l], gz);
+    }
+    g[a][0] = gx; g[a][1] = gy; g[a][2] = gz;
+  }
+  const double v13 = cbrt(V);
+  const double coef = -kappa * rho * c * v13 * v13;
+#pragma unroll
+  for (int l = 0; l < 8; ++l) {
+    double sx = 0.0, sy = 0.0, sz = 0.0;
+#pragma unroll
+    for (int a = 0; a < 4; ++a) {
+      sx = fma(gam[a][l], g[a][0], sx);
+      sy = fma(gam[a][l], g[a][1], sy);
+      sz = fma(gam[a][l], g[a][2], sz);
+    }
+    Fx[l] = fma(coef, sx, Fx[l]);
+    Fy[l] = fma(coef, sy, Fy[l]);
+    Fz[l] = fma(coef, sz, Fz[l]);
+  }
+}
+
 struct ZoneEos {
   double rho, p, c, q, P, dtz;
 };

@@ -22,7 +22,7 @@ LIB_PATH = os.environ.get("HYDRO_LIB") or os.path.join(_HERE, "libhydro_b200.so"
 NODE_FIELDS = ("x", "y", "z", "u", "v", "w")
 ZONE_FIELDS = ("rho", "e", "p", "q", "c", "vol", "mass")
 ALL_FIELDS = NODE_FIELDS + ZONE_FIELDS
-ABI_VERSION = 1
+ABI_VERSION = 2
 FLAG_NO_GRAPH = 1 << 0
 FLAG_SPLIT = 1 << 1
 FLAG_ONE_KERNEL = 1 << 2
@@ -53,6 +53,7 @@ class HydroConfigC(C.Structure):
         ("rank", C.c_int32), ("nranks", C.c_int32), ("device", C.c_int32),
         ("comm_id", C.c_void_p),
         ("flags", C.c_uint64),
+        ("hg_coef", C.c_double),
     ]
 
 
@@ -142,6 +143,8 @@ class HydroConfig:
     graph: bool = True            # CUDA graphs (HYDRO_FLAG_NO_GRAPH when False)
     transport: str = "nccl"       # nranks > 1: "nccl" (NCCL send/recv + allreduce) or "peer"
                                   # (CUDA IPC peer stores + mailbox reduction; ranks may share a GPU)
+    hg_coef: float = 0.0          # viscous hourglass kappa (reading R17); > 0 runs
+                                  # the split kernels
 
 
 class HydroError(RuntimeError):
@@ -172,7 +175,7 @@ def _cfg_struct(cfg: HydroConfig, keep: list, comm_id: Optional[bytes] = None) -
         keep.append(arr)
         c.rank_weight = arr.ctypes.data_as(C.POINTER(C.c_double))
     for k in ("gamma", "q_lin", "q_quad", "cfl", "c_vol", "dt_growth", "dt_max", "dt_init",
-              "t_stop", "dt_first", "t0", "rho0", "e0", "sedov_energy"):
+              "t_stop", "dt_first", "t0", "rho0", "e0", "sedov_energy", "hg_coef"):
         setattr(c, k, float(getattr(cfg, k)))
     c.reflect_mask = int(cfg.reflect_mask)
     c.init_kind = {"sedov": 0, "user": 1, "user_mass": 2}[cfg.init]
