@@ -167,6 +167,25 @@ int hydro_peer_import(hydro_ctx *h, const void *all, size_t len_per_rank);
 /* Current info without stepping. */
 int hydro_get_info(hydro_ctx *h, hydro_info *info);
 
+/* Domain migration: the complete state of one domain this rank owns, i.e.
+   its current node arrays x,y,z,u,v,w and zone arrays e and m over the domain's storage box
+   including the ghost layer (layout: 6 node arrays of (n0+3 padded to 4)(n1+3)(n2+3) doubles,
+   then e and m of (n0+2 padded to 4)(n1+2)(n2+2) doubles), as a flat device buffer.  The
+   storage depends only on the domain box, so a buffer packed by one context unpacks into any
+   context with the same cuts, on any rank; moving it between ranks is the caller's (e.g.
+   torch.distributed send/recv over NCCL).  hydro_domain_bytes: *len = bytes of dom's buffer
+   (host-only arithmetic, any domain).  pack: dev_buf (device, >= len bytes, caller-owned)
+   <- state, on `stream` (NULL = the context's), synchronised before return.  unpack: state <-
+   dev_buf, then 1/m and the nodal 8/sum m are recomputed for that domain.  Errors:
+   HYDRO_EINVAL (dom not owned by this rank, len too small), HYDRO_ECUDA. */
+int hydro_domain_bytes(const hydro_ctx *h, int32_t dom, size_t *len);
+int hydro_domain_pack(hydro_ctx *h, int32_t dom, void *dev_buf, size_t len, void *stream);
+int hydro_domain_unpack(hydro_ctx *h, int32_t dom, const void *dev_buf, size_t len,
+                        void *stream);
+/* Set the run clock (t, the dt of the next cycle, the cycle counter) and clear error state:
+   continues a migrated or restarted run exactly.  dt > 0.  Errors: HYDRO_EINVAL, HYDRO_ECUDA. */
+int hydro_set_clock(hydro_ctx *h, double t, double dt, int64_t cycle);
+
 /* Destroy; NULL-safe; collective. */
 int hydro_destroy(hydro_ctx *h);
 
@@ -209,6 +228,21 @@ int hydro_decompose_hierarchical(const int64_t n[3], int32_t ngpu, int32_t dpg, 
    nplanes planes over nparts parts with weights w: n_g = floor(N w_g / W), remaining planes to
    the largest remainders (ties: lowest g), every n_g >= 1.  out[nparts] receives n_g. */
 int hydro_weighted_slabs(int64_t nplanes, int32_t nparts, const double *w, int64_t *out);
+
+/* Measured-weight rebalancing between runs ("an initial
+   guess of work split ... based on FLOPS.  We measured the respective contributions ... and
+   adjusted the split"; L1077-1081: "static within an iteration, but the decomposition can be
+   adjusted between iterations").  Host-only and deterministic, so every rank computes the same
+   plan.  cfg describes the CURRENT layout (its dom_to_rank or weighted-rule map); busy[nranks]
+   is each rank's measured device time per cycle under it (> 0, any unit).  Domain cost =
+   owned zones + beta * ghost elements (beta >= 0, the surface term); rank speed
+   w_g = load_g / busy_g (normalised to mean 1; a rank without domains gets the mean); the new
+   map is the LPT rule with those weights (reading R19), kept only if the modelled makespan
+   max_g load_g / w_g drops by more than min_gain (fraction), else new_map = the current map.
+   Outputs: new_map[ndomains], weights[nranks] (may be NULL), predicted[2] = modelled makespan
+   before / after in busy units (may be NULL).  Errors: HYDRO_EINVAL. */
+int hydro_rebalance_plan(const hydro_config *cfg, const double *busy, double beta,
+                         double min_gain, int32_t *new_map, double *weights, double *predicted);
 
 /* 128-byte communicator id for nranks > 1 (call on rank 0, broadcast to all ranks). */
 int hydro_comm_unique_id(void *out128);

@@ -5,7 +5,9 @@ thin binding and ``inputs`` the seeded synthetic input generators.  Importing th
 not load the library; constructing ``Hydro`` does, and fails loudly if it is missing.
 """
 from .hydro import (ALL_FIELDS, Hydro, HydroConfig, HydroError, comm_plan_export,  # noqa
-                    decompose_hierarchical, layout_export, load_library, weighted_slabs)
+                    decompose_hierarchical, dom_to_rank, layout_export, load_library,
+                    rebalance_plan, weighted_slabs)
 
 __all__ = ["Hydro", "HydroConfig", "HydroError", "layout_export", "decompose_hierarchical",
-           "weighted_slabs", "load_library", "ALL_FIELDS", "comm_plan_export"]
+           "weighted_slabs", "load_library", "ALL_FIELDS", "comm_plan_export", "rebalance_plan",
+           "dom_to_rank"]

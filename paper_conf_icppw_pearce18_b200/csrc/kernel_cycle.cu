@@ -97,7 +97,6 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   // the chunked schedule (CTA b = column b / chunks, chunk b % chunks), for A/B measurement.
   int64_t r0, r1;
   if (sched_kz > 0) {
-    const int chunks = (n2 + sched_kz - 1) / sched_kz;
     const int64_t col = blockIdx.x % ncols, ch = blockIdx.x / ncols;  // adjacent CTAs: same z
     r0 = col * n2 + ch * sched_kz;
     r1 = col * n2 + min((int)(ch + 1) * sched_kz, n2);

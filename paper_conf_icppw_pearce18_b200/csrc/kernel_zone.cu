@@ -62,7 +62,6 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   const int64_t W = (int64_t)tcols * ((zhi.y - zlo.y + ZBY - 1) / ZBY) * nplanes;
   int64_t r0, r1;
   if (sched_kz > 0) {
-    const int chunks = (nplanes + sched_kz - 1) / sched_kz;
     const int ncols = tcols * ((zhi.y - zlo.y + ZBY - 1) / ZBY);
     const int64_t col = blockIdx.x % ncols, ch = blockIdx.x / ncols;  // adjacent CTAs: same z
     r0 = col * nplanes + ch * sched_kz;

@@ -221,6 +221,74 @@ int hydro_comm_plan_export(const hydro_config *cfg, int64_t *buf, size_t *len) {
   return (buf && cap < w.size()) ? HYDRO_EINVAL : HYDRO_OK;
 }
 
+int hydro_rebalance_plan(const hydro_config *cfg, const double *busy, double beta,
+                         double min_gain, int32_t *new_map, double *weights, double *predicted) {
+  if (!cfg || !busy || !new_map || !(beta >= 0.0) || !(min_gain >= 0.0)) return HYDRO_EINVAL;
+  Layout L;
+  std::string err;
+  const int rc = layout_build(cfg, &L, &err);
+  if (rc != HYDRO_OK) return rc;
+  const int nd = (int)L.dom.size(), G = cfg->nranks;
+  for (int g = 0; g < G; ++g)
+    if (!(busy[g] > 0.0) || !std::isfinite(busy[g])) return HYDRO_EINVAL;
+  // domain cost: owned zones + beta * ghost elements (the surface term)
+  std::vector<double> ghost(nd, 0.0);
+  for (const HaloPair &P : L.pairs) {
+    int64_t nn = 1, nz = 1;
+    for (int a = 0; a < 3; ++a) {
+      nn *= P.nhi[a] - P.nlo[a];
+      nz *= P.zhi[a] - P.zlo[a];
+    }
+    ghost[P.dst] += (double)(nn + nz);
+  }
+  std::vector<int64_t> cost(nd);
+  for (int d = 0; d < nd; ++d) {
+    const double c = (double)(L.dom[d].n[0] * L.dom[d].n[1] * L.dom[d].n[2]) + beta * ghost[d];
+    cost[d] = (int64_t)std::llround(c);
+  }
+  // measured speeds ("We measured the respective contributions ... and
+  // adjusted the split"): w_g = load_g / busy_g under the current map; a rank with no domain
+  // keeps the mean speed of the others
+  std::vector<double> load(G, 0.0), w(G, 0.0);
+  for (int d = 0; d < nd; ++d) load[L.dom[d].rank] += (double)cost[d];
+  double wsum = 0.0;
+  int nw = 0;
+  for (int g = 0; g < G; ++g)
+    if (load[g] > 0.0) {
+      w[g] = load[g] / busy[g];
+      wsum += w[g];
+      ++nw;
+    }
+  if (nw == 0) return HYDRO_EINVAL;
+  for (int g = 0; g < G; ++g)
+    if (!(load[g] > 0.0)) w[g] = wsum / nw;
+  double mean = 0.0;
+  for (int g = 0; g < G; ++g) mean += w[g];
+  mean /= G;
+  for (int g = 0; g < G; ++g) w[g] /= mean;
+  std::vector<int32_t> own = lpt_assign(cost, G, w.data());
+  // predicted makespans in the speed model (before = the measured map, after = LPT)
+  std::vector<double> l0(G, 0.0), l1(G, 0.0);
+  for (int d = 0; d < nd; ++d) {
+    l0[L.dom[d].rank] += (double)cost[d];
+    l1[own[d]] += (double)cost[d];
+  }
+  double before = 0.0, after = 0.0;
+  for (int g = 0; g < G; ++g) {
+    before = std::max(before, l0[g] / w[g]);
+    after = std::max(after, l1[g] / w[g]);
+  }
+  const bool move = after < before * (1.0 - min_gain);  // migration only for a real gain
+  for (int d = 0; d < nd; ++d) new_map[d] = move ? own[d] : L.dom[d].rank;
+  if (weights)
+    for (int g = 0; g < G; ++g) weights[g] = w[g];
+  if (predicted) {
+    predicted[0] = before;
+    predicted[1] = move ? after : before;
+  }
+  return HYDRO_OK;
+}
+
 int hydro_weighted_slabs(int64_t nplanes, int32_t nparts, const double *w, int64_t *out) {
   if (nparts < 1 || nplanes < nparts || !out) return HYDRO_EINVAL;
   double W = 0.0;

@@ -659,6 +659,92 @@ int hydro_get_info(hydro_ctx *h, hydro_info *info) {
   return HYDRO_OK;
 }
 
+namespace {
+// Storage sizes of a domain's migration buffer: 6 node arrays + e + m (hydro_domain_bytes).
+void domain_counts(const DomainBox &b, int64_t *nnode, int64_t *nzone) {
+  *nnode = (b.n[0] + 3 + 3) / 4 * 4 * (b.n[1] + 3) * (b.n[2] + 3);
+  *nzone = (b.n[0] + 2 + 3) / 4 * 4 * (b.n[1] + 2) * (b.n[2] + 2);
+}
+}  // namespace
+
+int hydro_domain_bytes(const hydro_ctx *h, int32_t dom, size_t *len) {
+  if (!h || !len || dom < 0 || dom >= (int32_t)h->L.dom.size()) return HYDRO_EINVAL;
+  int64_t nn, nz;
+  domain_counts(h->L.dom[dom], &nn, &nz);
+  *len = (size_t)(6 * nn + 2 * nz) * sizeof(double);
+  return HYDRO_OK;
+}
+
+int hydro_domain_pack(hydro_ctx *h, int32_t dom, void *dev_buf, size_t len, void *stream) {
+  size_t need = 0;
+  if (hydro_domain_bytes(h, dom, &need) || !dev_buf || len < need ||
+      h->slot_of_dom[dom] < 0)
+    return set_err(h, HYDRO_EINVAL, "domain_pack: bad domain, buffer or length");
+  CK(cudaSetDevice(h->device));
+  cudaStream_t s = stream ? (cudaStream_t)stream : h->stream;
+  const LocalDom &D = h->doms[h->slot_of_dom[dom]];
+  const DomView &v = D.view[h->parity];
+  int64_t nn, nz;
+  domain_counts(D.box, &nn, &nz);
+  const size_t nb = align_up(nn * sizeof(double), 256);
+  char *dst = (char *)dev_buf;
+  // the six current node arrays are consecutive allocations of pitch nb (carve_views)
+  CK(cudaMemcpy2DAsync(dst, nn * sizeof(double), v.x, nb, nn * sizeof(double), 6,
+                       cudaMemcpyDeviceToDevice, s));
+  dst += 6 * nn * sizeof(double);
+  CK(cudaMemcpyAsync(dst, v.e, nz * sizeof(double), cudaMemcpyDeviceToDevice, s));
+  dst += nz * sizeof(double);
+  CK(cudaMemcpyAsync(dst, v.m, nz * sizeof(double), cudaMemcpyDeviceToDevice, s));
+  CK(cudaStreamSynchronize(s));
+  return HYDRO_OK;
+}
+
+int hydro_domain_unpack(hydro_ctx *h, int32_t dom, const void *dev_buf, size_t len,
+                        void *stream) {
+  size_t need = 0;
+  if (hydro_domain_bytes(h, dom, &need) || !dev_buf || len < need ||
+      h->slot_of_dom[dom] < 0)
+    return set_err(h, HYDRO_EINVAL, "domain_unpack: bad domain, buffer or length");
+  CK(cudaSetDevice(h->device));
+  cudaStream_t s = stream ? (cudaStream_t)stream : h->stream;
+  const LocalDom &D = h->doms[h->slot_of_dom[dom]];
+  const DomView &v = D.view[h->parity];
+  int64_t nn, nz;
+  domain_counts(D.box, &nn, &nz);
+  const size_t nb = align_up(nn * sizeof(double), 256);
+  const char *src = (const char *)dev_buf;
+  CK(cudaMemcpy2DAsync(const_cast<double *>(v.x), nb, src, nn * sizeof(double), nn * sizeof(double), 6,
+                       cudaMemcpyDeviceToDevice, s));
+  src += 6 * nn * sizeof(double);
+  CK(cudaMemcpyAsync(const_cast<double *>(v.e), src, nz * sizeof(double), cudaMemcpyDeviceToDevice, s));
+  src += nz * sizeof(double);
+  CK(cudaMemcpyAsync(const_cast<double *>(v.m), src, nz * sizeof(double), cudaMemcpyDeviceToDevice, s));
+  launch_nodal_mass(D.view[0], s);  // 1/m and 8 / sum m from the imported masses
+  CK(cudaGetLastError());
+  CK(cudaStreamSynchronize(s));
+  return HYDRO_OK;
+}
+
+int hydro_set_clock(hydro_ctx *h, double t, double dt, int64_t cycle) {
+  if (!h || !(dt > 0.0) || !std::isfinite(t) || cycle < 0)
+    return set_err(h, HYDRO_EINVAL, "set_clock: bad argument");
+  CK(cudaSetDevice(h->device));
+  DevState s0;
+  CK(cudaMemcpyAsync(&s0, h->st, sizeof(s0), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  s0.t = t;
+  s0.dt = dt;
+  s0.cycle = (unsigned long long)cycle;
+  s0.err = 0;
+  s0.halted = 0;
+  s0.done = (h->ph.t_stop > 0.0 && t >= h->ph.t_stop) ? 1u : 0u;
+  s0.bad_zone = ~0ull;
+  CK(cudaMemcpyAsync(h->st, &s0, sizeof(s0), cudaMemcpyHostToDevice, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  h->failed = 0;
+  return HYDRO_OK;
+}
+
 int hydro_get_box(hydro_ctx *h, const int64_t lo[3], const int64_t hi[3], uint32_t mask,
                   double *const *out) {
   if (!h || !lo || !hi || !out) return set_err(h, HYDRO_EINVAL, "NULL argument");

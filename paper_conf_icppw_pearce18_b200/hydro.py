@@ -94,6 +94,13 @@ def load_library(path: str = LIB_PATH) -> C.CDLL:
                                          C.POINTER(C.c_size_t)]
     L.hydro_weighted_slabs.argtypes = [C.c_int64, C.c_int32, C.POINTER(C.c_double),
                                        C.POINTER(C.c_int64)]
+    L.hydro_rebalance_plan.argtypes = [C.POINTER(HydroConfigC), C.POINTER(C.c_double), C.c_double,
+                                       C.c_double, C.POINTER(C.c_int32), C.POINTER(C.c_double),
+                                       C.POINTER(C.c_double)]
+    L.hydro_domain_bytes.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_size_t)]
+    L.hydro_domain_pack.argtypes = [C.c_void_p, C.c_int32, C.c_void_p, C.c_size_t, C.c_void_p]
+    L.hydro_domain_unpack.argtypes = [C.c_void_p, C.c_int32, C.c_void_p, C.c_size_t, C.c_void_p]
+    L.hydro_set_clock.argtypes = [C.c_void_p, C.c_double, C.c_double, C.c_int64]
     L.hydro_comm_unique_id.argtypes = [C.c_void_p]
     L.hydro_peer_export.argtypes = [C.c_void_p, C.c_void_p, C.POINTER(C.c_size_t)]
     L.hydro_peer_import.argtypes = [C.c_void_p, C.c_void_p, C.c_size_t]
@@ -254,6 +261,35 @@ def weighted_slabs(nplanes: int, weights: Sequence[float]):
     return out.tolist()
 
 
+def rebalance_plan(cfg: HydroConfig, busy: Sequence[float], beta: float = 0.0,
+                   min_gain: float = 0.02):
+    """hydro_rebalance_plan (host-only): (new dom_to_rank, rank speeds, (before, after))."""
+    L = load_library()
+    keep: list = []
+    c = _cfg_struct(cfg, keep)
+    nd = int(cfg.ndom[0]) * int(cfg.ndom[1]) * int(cfg.ndom[2])
+    b = np.ascontiguousarray(busy, dtype=np.float64)
+    if b.size != cfg.nranks:
+        raise ValueError("busy needs one entry per rank")
+    new_map = np.zeros(nd, dtype=np.int32)
+    w = np.zeros(cfg.nranks, dtype=np.float64)
+    pred = np.zeros(2, dtype=np.float64)
+    rc = L.hydro_rebalance_plan(C.byref(c), b.ctypes.data_as(C.POINTER(C.c_double)),
+                                float(beta), float(min_gain),
+                                new_map.ctypes.data_as(C.POINTER(C.c_int32)),
+                                w.ctypes.data_as(C.POINTER(C.c_double)),
+                                pred.ctypes.data_as(C.POINTER(C.c_double)))
+    if rc != 0:
+        raise HydroError(rc, "rebalance_plan")
+    return new_map.tolist(), w.tolist(), (float(pred[0]), float(pred[1]))
+
+
+def dom_to_rank(cfg: HydroConfig):
+    """The domain -> rank map cfg resolves to (explicit map or the weighted LPT rule)."""
+    lay = layout_export(cfg).tolist()
+    return [int(lay[7 + 7 * d + 6]) for d in range(int(lay[1]))]
+
+
 def _info(i: HydroInfoC) -> dict:
     return {"t": i.t, "dt": i.dt, "cycle": i.cycle, "dt_min_zone": i.dt_min_zone,
             "status": i.status, "bad_zone": i.bad_zone}
@@ -263,9 +299,12 @@ class Hydro:
     """One hydro run on this process's GPU (collective over ranks when nranks > 1)."""
 
     def __init__(self, cfg: HydroConfig, group=None):
-        self.cfg = cfg
         self._L = load_library()
         self._group = group
+        self._create(cfg)
+
+    def _create(self, cfg: HydroConfig):
+        self.cfg = cfg
         comm_id = None
         if cfg.nranks > 1 and cfg.transport == "nccl":
             comm_id = self._bootstrap_comm_id()
@@ -393,6 +432,97 @@ class Hydro:
                 t = t.cuda()
             dist.all_reduce(t, group=self._group)  # each entry is written by exactly one rank
             res[k] = t.cpu().numpy()
+        return res
+
+    # ------------------------------------------------------------ domain migration (f2)
+    def domain_bytes(self, dom: int) -> int:
+        n = C.c_size_t(0)
+        rc = self._L.hydro_domain_bytes(self._h, int(dom), C.byref(n))
+        if rc != 0:
+            raise HydroError(rc, "domain_bytes")
+        return int(n.value)
+
+    def pack_domain(self, dom: int):
+        """hydro_domain_pack into a new CUDA uint8 tensor (this rank must own ``dom``)."""
+        import torch
+        buf = torch.empty(self.domain_bytes(dom), dtype=torch.uint8,
+                          device=f"cuda:{self.cfg.device}")
+        rc = self._L.hydro_domain_pack(self._h, int(dom), C.c_void_p(buf.data_ptr()), buf.numel(),
+                                       None)
+        if rc != 0:
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+        return buf
+
+    def unpack_domain(self, dom: int, buf):
+        rc = self._L.hydro_domain_unpack(self._h, int(dom), C.c_void_p(buf.data_ptr()),
+                                         buf.numel(), None)
+        if rc != 0:
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+
+    def set_clock(self, t: float, dt: float, cycle: int):
+        rc = self._L.hydro_set_clock(self._h, float(t), float(dt), int(cycle))
+        if rc != 0:
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+
+    def rebalance(self, busy: Optional[Sequence[float]] = None, beta: float = 0.0,
+                  min_gain: float = 0.02, measure_cycles: int = 5) -> dict:
+        """Measured-weight rebalancing between iterations (PAPER.md L597-603,
+        L1077-1081).  Collective.  busy: per-rank device ms per cycle under the current map;
+        None = measure it here with hydro_time_kernels over ``measure_cycles`` cycles (real
+        cycles: the run advances) and all-gather it.  The plan is hydro_rebalance_plan; domains
+        whose owner changes are packed on the old owner, sent with torch.distributed (device
+        tensors over NCCL, host copies over gloo) and unpacked into a new context built with the
+        new map; the clock carries over, so the run continues exactly."""
+        import dataclasses
+        import torch
+        import torch.distributed as dist
+        cfg = self.cfg
+        cur = dom_to_rank(cfg)
+        if busy is None:
+            own = self.time_kernels(measure_cycles)["cycle_kernel_ms"]
+            if cfg.nranks > 1:
+                allb = [None] * cfg.nranks
+                dist.all_gather_object(allb, own, group=self._group)
+                busy = allb
+            else:
+                busy = [own]
+        cur_cfg = dataclasses.replace(cfg, dom_to_rank=cur, rank_weight=None)
+        new_map, weights, pred = rebalance_plan(cur_cfg, busy, beta, min_gain)
+        res = {"map": new_map, "weights": weights, "predicted": pred, "busy": list(busy),
+               "moved": sum(int(a != b) for a, b in zip(cur, new_map))}
+        if res["moved"] == 0:
+            return res
+        info = self.info()
+        rank = cfg.rank
+        bufs = {d: self.pack_domain(d) for d in range(len(cur)) if cur[d] == rank}
+        if cfg.nranks > 1:
+            host = dist.get_backend(self._group) != "nccl"
+            ops, recvd = [], {}
+            for d in range(len(cur)):
+                a, b = cur[d], new_map[d]
+                if a == b:
+                    continue
+                if a == rank:
+                    t = bufs[d].cpu() if host else bufs[d]
+                    ops.append(dist.P2POp(dist.isend, t, b, group=self._group))
+                if b == rank:
+                    n = self.domain_bytes(d)
+                    t = torch.empty(n, dtype=torch.uint8,
+                                    device="cpu" if host else f"cuda:{cfg.device}")
+                    recvd[d] = t
+                    ops.append(dist.P2POp(dist.irecv, t, a, group=self._group))
+            if ops:
+                for r in dist.batch_isend_irecv(ops):
+                    r.wait()
+            for d, t in recvd.items():
+                bufs[d] = t.to(f"cuda:{cfg.device}")
+        self.close()
+        self._create(dataclasses.replace(cfg, dom_to_rank=new_map, rank_weight=None))
+        for d in range(len(new_map)):
+            if new_map[d] == rank:
+                self.unpack_domain(d, bufs[d])
+        del bufs
+        self.set_clock(info["t"], info["dt"], info["cycle"])
         return res
 
     def set_state(self, nodes: Dict[str, np.ndarray], e: np.ndarray, t: float, dt: float):
