@@ -70,6 +70,13 @@ enum : unsigned int { ERR_TANGLED = 1u, ERR_NONFINITE = 2u };
 // S9: t' = t + dt, dt' = min(min(growth*dt, dt_max), min_z dt_z), t_stop clamp;
 // latch the cycle's error bits so later cycles become no-ops (the state stays the one after the
 // failing cycle, as in the oracle).  Run by one thread after every kernel of the cycle.
+// PDL (kernels.h launch_pdl): wait for the preceding kernel's completion and memory flush, then
+// let the next kernel launch.  No-ops when the kernel was launched without the attribute.
+__device__ __forceinline__ void pdl_wait_and_trigger() {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 __device__ __forceinline__ void finalize_cycle(DevState *st, const Phys &ph) {
   if (st->halted | st->done) return;
   const double dtmin = __longlong_as_double((long long)st->dtz_acc);

@@ -83,6 +83,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   uint64_t *bar = reinterpret_cast<uint64_t *>(sm + T::OFF_BAR);
   constexpr int ZS = T::ZS, RS = T::RS, TXT = T::TXT, ZRS = T::ZRS, PX = T::PX;
 
+  pdl_wait_and_trigger();
   const int t = threadIdx.x;
   const int n0 = d.n[0], n1 = d.n[1], n2 = d.n[2];
   // lanes: zone/node (tx, ty) for tx < TXT; tx == TXT forms the box's last node column; the
@@ -558,7 +559,8 @@ void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st
   } else {
     G = (int)std::min<int64_t>(sms, (int64_t)ncols * d.n[2]);
   }
-  k_cycle<CTX, CTY, FUSED><<<G, T::NTHR, T::BYTES, s>>>(maps, d, ph, st, tx, ncols, kz, fold);
+  launch_pdl(k_cycle<CTX, CTY, FUSED>, dim3(G), dim3(T::NTHR), T::BYTES, s, maps, d, ph, st, tx,
+             ncols, kz, fold);
 }
 
 }  // namespace

@@ -53,6 +53,7 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   extern __shared__ __align__(1024) double sm[];
   double *RAW = sm + ZOFF_RAW, *XP = sm + ZOFF_XP;
   uint64_t *bar = reinterpret_cast<uint64_t *>(sm + ZOFF_BAR);
+  pdl_wait_and_trigger();
   if ((st->halted | st->done) != 0u) return;
 
   const int t = threadIdx.x;
@@ -298,8 +299,8 @@ void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, D
   } else {
     G = (int)std::min<int64_t>(slots, units);
   }
-  k_zone_stage<<<G, ZBX * ZBY, ZBYTES, s>>>(maps, d, ph, st, tx, kz, lo[0], lo[1], lo[2], hi[0],
-                                            hi[1], hi[2]);
+  launch_pdl(k_zone_stage, dim3(G), dim3(ZBX * ZBY), ZBYTES, s, maps, d, ph, st, tx, kz, lo[0],
+             lo[1], lo[2], hi[0], hi[1], hi[2]);
 }
 
 }  // namespace hydro

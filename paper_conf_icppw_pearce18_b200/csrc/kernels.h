@@ -10,10 +10,35 @@
 
 namespace hydro {
 
-struct HaloCopy {  // one intra-GPU ghost slab copy (global boxes, half-open)
+// Programmatic dependent launch (PDL): the per-cycle kernels are launched with
+// cudaLaunchAttributeProgrammaticStreamSerialization, start `griddepcontrol.wait` (pdl_wait in
+// device.cuh) before touching global memory, and trigger their dependents right after, so the
+// next kernel's CTAs are launched and set up while this one drains (CUDA graphs keep the
+// programmatic edges).  HYDRO_NO_PDL=1 launches them plainly (A/B measurement).
+bool pdl_enabled();
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                       Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
+}
+
+struct HaloCopy {  // one chunk of an intra-GPU ghost slab copy (global boxes, half-open)
   int32_t dst, src;  // local domain slots
   int64_t nlo[3], nhi[3], zlo[3], zhi[3];
+  int32_t kind;         // 0: the node slab (x,y,z,u,v,w), 1: the zone slab (e)
+  int32_t start, count; // elements [start, start+count) of that slab, x fastest
 };
+constexpr int HALO_CHUNK = 2048;  // elements per chunk (one CTA of 256 threads)
 
 // Initialisation.
 void launch_init_nodes(const DomView &d, const double origin[3], const double extent[3],
@@ -66,8 +91,8 @@ int cycle_zone_box_y();
 void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s);
 
 // Intra-GPU ghost exchange of the next-parity state over a table of slab copies.
-void launch_halo_copy(const DomView *views_dev, const HaloCopy *pairs_dev, int npairs,
-                      int blocks_per_pair, cudaStream_t s);
+void launch_halo_copy(const DomView *views_dev, const HaloCopy *chunks_dev, int nchunks,
+                      cudaStream_t s);
 
 // Strided 3-D box copy (src/dst pre-offset to the box origin; pitches in elements).
 void launch_copy3d(const double *src, int64_t ssx, int64_t ssxy, double *dst, int64_t dsx,

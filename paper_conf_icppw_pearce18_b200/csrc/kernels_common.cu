@@ -151,7 +151,10 @@ __global__ void k_finalize_init(DevState *st, double dt_first, double dt_init, d
 }
 
 // S9 as its own kernel (multi-domain / multi-rank cycles; see finalize_cycle).
-__global__ void k_finalize(DevState *st, Phys ph) { finalize_cycle(st, ph); }
+__global__ void k_finalize(DevState *st, Phys ph) {
+  pdl_wait_and_trigger();
+  finalize_cycle(st, ph);
+}
 
 // ------------------------------------------------------------------ split pipeline
 // K1: S1-S6 for every existing local zone (owned and ghost): P and the 24 corner-vector
@@ -269,39 +272,41 @@ __global__ void k_energy_split(DomView d, Phys ph, DevState *st) {
 }
 
 // ---------------------------------------------------------------------- halo copy
-__global__ void k_halo_copy(const DomView *views, const HaloCopy *pairs) {
-  const HaloCopy p = pairs[blockIdx.y];
+__global__ void k_halo_copy(const DomView *views, const HaloCopy *chunks) {
+  // one CTA per chunk of HALO_CHUNK slab elements (host-built list): no idle CTAs
+  // for the many small edge and corner slabs.  32-bit index arithmetic (slabs and domain storage
+  // are below 2^31 elements).
+  const HaloCopy p = chunks[blockIdx.x];
   const DomView &D = views[p.dst];
   const DomView &S = views[p.src];
-  // 32-bit index arithmetic (slabs and domain storage are below 2^31 elements)
-  const int nx = (int)(p.nhi[0] - p.nlo[0]), ny = (int)(p.nhi[1] - p.nlo[1]);
-  const int nn = nx * ny * (int)(p.nhi[2] - p.nlo[2]);
-  // local node index of the slab origin in both domains; element (a, b, c) is origin + offsets
-  const int dsx = (int)D.nsx, dsxy = (int)D.nsxy, ssx = (int)S.nsx, ssxy = (int)S.nsxy;
-  const int d0 = (int)D.nid((int)(p.nlo[0] - D.lo[0]), (int)(p.nlo[1] - D.lo[1]),
-                            (int)(p.nlo[2] - D.lo[2]));
-  const int s0 = (int)S.nid((int)(p.nlo[0] - S.lo[0]), (int)(p.nlo[1] - S.lo[1]),
-                            (int)(p.nlo[2] - S.lo[2]));
-  for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < nn; t += gridDim.x * blockDim.x) {
-    const int a = t % nx, r = t / nx, b = r % ny, c = r / ny;
-    const int di = d0 + c * dsxy + b * dsx + a, si = s0 + c * ssxy + b * ssx + a;
-    D.xn[di] = S.xn[si];
-    D.yn[di] = S.yn[si];
-    D.zn[di] = S.zn[si];
-    D.un[di] = S.un[si];
-    D.vn[di] = S.vn[si];
-    D.wn[di] = S.wn[si];
-  }
-  const int zx = (int)(p.zhi[0] - p.zlo[0]), zy = (int)(p.zhi[1] - p.zlo[1]);
-  const int nzn = zx * zy * (int)(p.zhi[2] - p.zlo[2]);
-  const int zdsx = (int)D.zsx, zdsxy = (int)D.zsxy, zssx = (int)S.zsx, zssxy = (int)S.zsxy;
-  const int zd0 = (int)D.zid((int)(p.zlo[0] - D.lo[0]), (int)(p.zlo[1] - D.lo[1]),
-                             (int)(p.zlo[2] - D.lo[2]));
-  const int zs0 = (int)S.zid((int)(p.zlo[0] - S.lo[0]), (int)(p.zlo[1] - S.lo[1]),
-                             (int)(p.zlo[2] - S.lo[2]));
-  for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < nzn; t += gridDim.x * blockDim.x) {
-    const int a = t % zx, r = t / zx, b = r % zy, c = r / zy;
-    D.en[zd0 + c * zdsxy + b * zdsx + a] = S.en[zs0 + c * zssxy + b * zssx + a];
+  if (p.kind == 0) {
+    const int nx = (int)(p.nhi[0] - p.nlo[0]), ny = (int)(p.nhi[1] - p.nlo[1]);
+    const int dsx = (int)D.nsx, dsxy = (int)D.nsxy, ssx = (int)S.nsx, ssxy = (int)S.nsxy;
+    const int d0 = (int)D.nid((int)(p.nlo[0] - D.lo[0]), (int)(p.nlo[1] - D.lo[1]),
+                              (int)(p.nlo[2] - D.lo[2]));
+    const int s0 = (int)S.nid((int)(p.nlo[0] - S.lo[0]), (int)(p.nlo[1] - S.lo[1]),
+                              (int)(p.nlo[2] - S.lo[2]));
+    for (int t = p.start + threadIdx.x; t < p.start + p.count; t += blockDim.x) {
+      const int a = t % nx, r = t / nx, b = r % ny, c = r / ny;
+      const int di = d0 + c * dsxy + b * dsx + a, si = s0 + c * ssxy + b * ssx + a;
+      D.xn[di] = S.xn[si];
+      D.yn[di] = S.yn[si];
+      D.zn[di] = S.zn[si];
+      D.un[di] = S.un[si];
+      D.vn[di] = S.vn[si];
+      D.wn[di] = S.wn[si];
+    }
+  } else {
+    const int zx = (int)(p.zhi[0] - p.zlo[0]), zy = (int)(p.zhi[1] - p.zlo[1]);
+    const int zdsx = (int)D.zsx, zdsxy = (int)D.zsxy, zssx = (int)S.zsx, zssxy = (int)S.zsxy;
+    const int zd0 = (int)D.zid((int)(p.zlo[0] - D.lo[0]), (int)(p.zlo[1] - D.lo[1]),
+                               (int)(p.zlo[2] - D.lo[2]));
+    const int zs0 = (int)S.zid((int)(p.zlo[0] - S.lo[0]), (int)(p.zlo[1] - S.lo[1]),
+                               (int)(p.zlo[2] - S.lo[2]));
+    for (int t = p.start + threadIdx.x; t < p.start + p.count; t += blockDim.x) {
+      const int a = t % zx, r = t / zx, b = r % zy, c = r / zy;
+      D.en[zd0 + c * zdsxy + b * zdsx + a] = S.en[zs0 + c * zssxy + b * zssx + a];
+    }
   }
 }
 
@@ -372,13 +377,18 @@ void launch_node_split(const DomView &d, const Phys &ph, DevState *st, cudaStrea
 void launch_energy_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
   k_energy_split<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph, st);
 }
-void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s) {
-  k_finalize<<<1, 1, 0, s>>>(st, ph);
+bool pdl_enabled() {
+  static const int on = getenv("HYDRO_NO_PDL") && atoi(getenv("HYDRO_NO_PDL")) ? 0 : 1;
+  return on != 0;
 }
-void launch_halo_copy(const DomView *views_dev, const HaloCopy *pairs_dev, int npairs,
-                      int blocks_per_pair, cudaStream_t s) {
-  if (npairs <= 0) return;
-  k_halo_copy<<<dim3(blocks_per_pair, npairs), 256, 0, s>>>(views_dev, pairs_dev);
+
+void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s) {
+  launch_pdl(k_finalize, dim3(1), dim3(1), 0, s, st, ph);
+}
+void launch_halo_copy(const DomView *views_dev, const HaloCopy *chunks_dev, int nchunks,
+                      cudaStream_t s) {
+  if (nchunks <= 0) return;
+  k_halo_copy<<<nchunks, 256, 0, s>>>(views_dev, chunks_dev);
 }
 void launch_copy3d(const double *src, int64_t ssx, int64_t ssxy, double *dst, int64_t dsx,
                    int64_t dsxy, int ex, int ey, int ez, cudaStream_t s) {

@@ -50,7 +50,6 @@ struct hydro_ctx {
   DomView *views_dev[2] = {nullptr, nullptr};
   HaloCopy *local_pairs_dev = nullptr;
   int n_local_pairs = 0;
-  int halo_blocks = 1;  // blocks per intra-GPU halo slab (sized by the largest slab)
   cudaGraphExec_t graph[2] = {nullptr, nullptr};
   int parity = 0;
   bool split = false;
@@ -328,7 +327,7 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
     }
     for (LocalDom &D : h->doms) launch_node_stage(h, D, par, s);
   }
-  launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, h->halo_blocks, s);
+  launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
   if (h->comm) {
     int rc = comm_halo(h->comm, par, s);
     if (rc) return set_err(h, rc, "halo exchange failed");
@@ -530,22 +529,27 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
              HaloCopy c;
              c.dst = h->slot_of_dom[P.dst];
              c.src = h->slot_of_dom[P.src];
+             int64_t nn = 1, nz = 1;
              for (int a = 0; a < 3; ++a) {
                c.nlo[a] = P.nlo[a]; c.nhi[a] = P.nhi[a]; c.zlo[a] = P.zlo[a]; c.zhi[a] = P.zhi[a];
+               nn *= P.nhi[a] - P.nlo[a];
+               nz *= P.zhi[a] - P.zlo[a];
              }
-             lp.push_back(c);
+             // chunks of HALO_CHUNK elements: the node slab, then the zone slab
+             for (int kind = 0; kind < 2; ++kind) {
+               const int64_t total = kind ? nz : nn;
+               for (int64_t st = 0; st < total; st += HALO_CHUNK) {
+                 c.kind = kind;
+                 c.start = (int32_t)st;
+                 c.count = (int32_t)std::min<int64_t>(HALO_CHUNK, total - st);
+                 lp.push_back(c);
+               }
+             }
            } else if (dst_local || src_local) {
              remote.push_back(P);
            }
          }
-         h->n_local_pairs = (int)lp.size();
-         int64_t biggest = 0;
-         for (const HaloCopy &c : lp) {
-           int64_t nn = 1;
-           for (int a = 0; a < 3; ++a) nn *= c.nhi[a] - c.nlo[a];
-           biggest = std::max(biggest, nn);
-         }
-         h->halo_blocks = (int)std::max<int64_t>(1, std::min<int64_t>(1024, biggest / 1024));
+         h->n_local_pairs = (int)lp.size();  // chunk entries
          if (!lp.empty()) {
            CK(cudaMalloc(&h->local_pairs_dev, sizeof(HaloCopy) * lp.size()));
            CK(cudaMemcpyAsync(h->local_pairs_dev, lp.data(), sizeof(HaloCopy) * lp.size(),
@@ -886,7 +890,7 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
       for (LocalDom &D : h->doms) launch_node_stage(h, D, par, s);
     }
     CK(cudaEventRecord(ev[1], s));
-    launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, h->halo_blocks, s);
+    launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
     if (h->comm && comm_halo(h->comm, par, s)) return HYDRO_ENCCL;
     if (h->peer && peer_exchange(h->peer, h->views_dev[par], par, true, h->st, s))
       return HYDRO_ECUDA;
