@@ -70,10 +70,13 @@ struct CTile {
   static_assert(BYTES <= 227 * 1024, "shared memory");
 };
 
-template <int TX, int TY, bool FUSED>
+// GROUP: one chunked launch over all domains of this GPU; CTA b belongs to the NodeTask whose
+// [cta0, cta0 + ctas) contains b (adjacent CTAs: adjacent columns of one domain, same z-chunk).
+template <int TX, int TY, bool FUSED, bool GROUP>
 __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
-    k_cycle(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st, int tcols,
-            int ncols, int sched_kz, int fold_finalize) {
+    k_cycle(const __grid_constant__ NodeMaps maps1, const __grid_constant__ DomView d1, Phys ph,
+            DevState *st, int tcols1, int ncols1, int sched_kz1, int fold_finalize,
+            const NodeTask *tasks, int ntasks, const DomView *views, const NodeMaps *mapsg) {
   using T = CTile<TX, TY>;
   // dynamic shared memory only (no static __shared__), so the window is 1024-byte aligned
   extern __shared__ __align__(1024) double sm[];
@@ -84,6 +87,15 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   constexpr int ZS = T::ZS, RS = T::RS, TXT = T::TXT, ZRS = T::ZRS, PX = T::PX;
 
   pdl_wait_and_trigger();
+  int task_i = 0;
+  if (GROUP)
+    while (task_i + 1 < ntasks && (int)blockIdx.x >= tasks[task_i + 1].cta0) ++task_i;
+  const DomView &d = GROUP ? views[tasks[task_i].slot] : d1;
+  const NodeMaps &maps = GROUP ? mapsg[tasks[task_i].slot] : maps1;
+  const int ncols = GROUP ? tasks[task_i].ncols : ncols1;
+  const int tcols = GROUP ? tasks[task_i].tcols : tcols1;
+  const int sched_kz = GROUP ? tasks[task_i].kz : sched_kz1;
+  const int bid = GROUP ? (int)blockIdx.x - tasks[task_i].cta0 : (int)blockIdx.x;
   const int t = threadIdx.x;
   const int n0 = d.n[0], n1 = d.n[1], n2 = d.n[2];
   // lanes: zone/node (tx, ty) for tx < TXT; tx == TXT forms the box's last node column; the
@@ -98,7 +110,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   // the chunked schedule (CTA b = column b / chunks, chunk b % chunks), for A/B measurement.
   int64_t r0, r1;
   if (sched_kz > 0) {
-    const int64_t col = blockIdx.x % ncols, ch = blockIdx.x / ncols;  // adjacent CTAs: same z
+    const int64_t col = bid % ncols, ch = bid / ncols;  // adjacent CTAs: same z
     r0 = col * n2 + ch * sched_kz;
     r1 = col * n2 + min((int)(ch + 1) * sched_kz, n2);
   } else {
@@ -533,17 +545,35 @@ int choose_kz(int tiles, int n2, int sms) {
 }
 
 template <bool FUSED>
-void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st, int fold,
-            cudaStream_t s) {
-  using T = CTile<CTX, CTY>;
+void set_smem() {
+  static bool done = false;
+  if (!done) {
+    using T = CTile<CTX, CTY>;
+    cudaFuncSetAttribute(k_cycle<CTX, CTY, FUSED, false>,
+                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)T::BYTES);
+    if constexpr (!FUSED)
+      cudaFuncSetAttribute(k_cycle<CTX, CTY, false, true>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)T::BYTES);
+    done = true;
+  }
+}
+
+int num_sms() {
   static int sms = 0;
   if (!sms) {
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaFuncSetAttribute(k_cycle<CTX, CTY, FUSED>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)T::BYTES);
   }
+  return sms;
+}
+
+template <bool FUSED>
+void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st, int fold,
+            cudaStream_t s) {
+  using T = CTile<CTX, CTY>;
+  set_smem<FUSED>();
+  const int sms = num_sms();
   const int tx = (d.n[0] + CTX - 1) / CTX, ty = (d.n[1] + CTY - 1) / CTY;
   // Default: the chunked schedule (CTAs adjacent in x, y at the same z-chunk, so the tile rings
   // that neighbouring CTAs both read are L2 hits; measured faster here than the persistent
@@ -559,8 +589,9 @@ void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st
   } else {
     G = (int)std::min<int64_t>(sms, (int64_t)ncols * d.n[2]);
   }
-  launch_pdl(k_cycle<CTX, CTY, FUSED>, dim3(G), dim3(T::NTHR), T::BYTES, s, maps, d, ph, st, tx,
-             ncols, kz, fold);
+  launch_pdl(k_cycle<CTX, CTY, FUSED, false>, dim3(G), dim3(T::NTHR), T::BYTES, s, maps, d, ph,
+             st, tx, ncols, kz, fold, (const NodeTask *)nullptr, 0, (const DomView *)nullptr,
+             (const NodeMaps *)nullptr);
 }
 
 }  // namespace
@@ -579,6 +610,51 @@ void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, 
 void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                         int fold_finalize, cudaStream_t s) {
   launch<false>(d, maps, ph, st, fold_finalize, s);
+}
+
+int node_group_tasks(const DomView *views_host, int n, NodeTask *out) {
+  // one z-chunk length for all domains: minimise (waves of all CTAs) x (chunk + 2 warm-up
+  // planes) over the concatenated grid, as choose_kz does for one domain
+  const int sms = num_sms();
+  int nzmax = 1;
+  for (int i = 0; i < n; ++i) nzmax = std::max(nzmax, views_host[i].n[2]);
+  int best = nzmax, best_cost = INT_MAX;
+  for (int kz = 4; kz <= nzmax; ++kz) {
+    int64_t ctas = 0;
+    for (int i = 0; i < n; ++i) {
+      const DomView &d = views_host[i];
+      const int cols = ((d.n[0] + CTX - 1) / CTX) * ((d.n[1] + CTY - 1) / CTY);
+      ctas += (int64_t)cols * ((d.n[2] + kz - 1) / kz);
+    }
+    const int64_t cost = ((ctas + sms - 1) / sms) * (kz + 2);
+    if (cost < best_cost) {
+      best_cost = (int)cost;
+      best = kz;
+    }
+  }
+  int cta = 0;
+  for (int i = 0; i < n; ++i) {
+    const DomView &d = views_host[i];
+    NodeTask &T = out[i];
+    T.slot = i;
+    T.tcols = (d.n[0] + CTX - 1) / CTX;
+    T.ncols = T.tcols * ((d.n[1] + CTY - 1) / CTY);
+    T.kz = std::min(best, d.n[2]);
+    T.cta0 = cta;
+    cta += T.ncols * ((d.n[2] + T.kz - 1) / T.kz);
+  }
+  return cta;
+}
+
+void launch_node_energy_group(const NodeTask *tasks_dev, int ntasks, int nctas,
+                              const DomView *views_dev, const NodeMaps *maps_dev, const Phys &ph,
+                              DevState *st, cudaStream_t s) {
+  using T = CTile<CTX, CTY>;
+  set_smem<false>();
+  DomView d0 = {};
+  NodeMaps m0 = {};
+  launch_pdl(k_cycle<CTX, CTY, false, true>, dim3(nctas), dim3(T::NTHR), T::BYTES, s, m0, d0,
+             ph, st, 0, 0, 0, 0, tasks_dev, ntasks, views_dev, maps_dev);
 }
 
 }  // namespace hydro

@@ -43,13 +43,16 @@ static_assert(ZNX >= ZBX + 2, "zone-kernel TMA box too narrow (33 nodes + 1 alig
 // CTA b of G takes the contiguous range [b W / G, (b+1) W / G) and marches it as one or two
 // column segments (a range may cross a column boundary), so every CTA does the same number of
 // planes (plus one pipeline warm-up plane per segment) and the grid is exactly one wave.
-// sched_kz > 0 selects the chunked schedule instead (CTA b = column b / chunks, chunk b % chunks
-// of sched_kz planes), kept for A/B measurement.
+// GROUP: the units of ALL domains of this GPU are concatenated (ZoneTask table, u0 = prefix), so
+// one launch covers every domain and small domains share the SMs instead of each running a
+// short, tail-dominated grid.  sched_kz > 0 (single domain only) selects the chunked schedule
+// instead (CTA b = column b % ncols, chunk b / ncols of sched_kz planes), kept for A/B.
+template <bool GROUP>
 __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
-    k_zone_stage(const __grid_constant__ NodeMaps maps, DomView d, Phys ph, DevState *st,
-                 int tcols, int sched_kz, int zlox, int zloy, int zloz, int zhix, int zhiy,
-                 int zhiz) {
-  const int3 zlo = make_int3(zlox, zloy, zloz), zhi = make_int3(zhix, zhiy, zhiz);
+    k_zone_stage(const __grid_constant__ NodeMaps maps1, const __grid_constant__ DomView d1,
+                 const __grid_constant__ ZoneTask task1, const DomView *views,
+                 const NodeMaps *mapsg, const ZoneTask *tasks, int64_t Wtot, int sched_kz,
+                 Phys ph, DevState *st) {
   extern __shared__ __align__(1024) double sm[];
   double *RAW = sm + ZOFF_RAW, *XP = sm + ZOFF_XP;
   uint64_t *bar = reinterpret_cast<uint64_t *>(sm + ZOFF_BAR);
@@ -58,22 +61,19 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
 
   const int t = threadIdx.x;
   const int tx = t % ZBX, ty = t / ZBX;
-  const int n0 = d.n[0], n1 = d.n[1], n2 = d.n[2];
-  const int nplanes = zhi.z - zlo.z;
-  const int64_t W = (int64_t)tcols * ((zhi.y - zlo.y + ZBY - 1) / ZBY) * nplanes;
   int64_t r0, r1;
-  if (sched_kz > 0) {
-    const int ncols = tcols * ((zhi.y - zlo.y + ZBY - 1) / ZBY);
+  if (!GROUP && sched_kz > 0) {
+    const int nplanes = task1.zhi[2] - task1.zlo[2];
+    const int ncols = (int)(task1.units / nplanes);
     const int64_t col = blockIdx.x % ncols, ch = blockIdx.x / ncols;  // adjacent CTAs: same z
     r0 = col * nplanes + ch * sched_kz;
     r1 = col * nplanes + min((int)(ch + 1) * sched_kz, nplanes);
   } else {
-    r0 = W * blockIdx.x / gridDim.x;
-    r1 = W * (blockIdx.x + 1) / gridDim.x;
+    r0 = Wtot * blockIdx.x / gridDim.x;
+    r1 = Wtot * (blockIdx.x + 1) / gridDim.x;
   }
   const double dt = st->dt;
   const double hh = 0.5 * dt;
-  const int gz_lo = -(int)d.lo[2], gz_hi = d.N[2] - (int)d.lo[2];
   const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
   double dt2min = INFINITY;
   uint32_t ubase = 0;  // planes this CTA consumed in earlier segments (mbarrier phase continuity)
@@ -85,11 +85,24 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   }
   __syncthreads();
 
+  int ti = 0;  // current task (GROUP)
   for (int64_t r = r0; r < r1;) {
-    const int col = (int)(r / nplanes);
-    const int zk0 = zlo.z + (int)(r - (int64_t)col * nplanes);
-    const int zk1 = zlo.z + (int)min((int64_t)nplanes, r1 - (int64_t)col * nplanes);
-    r = (int64_t)col * nplanes + (zk1 - zlo.z);
+    if (GROUP)
+      while (r >= tasks[ti].u0 + tasks[ti].units) ++ti;
+    const ZoneTask &T = GROUP ? tasks[ti] : task1;
+    const DomView &d = GROUP ? views[T.slot] : d1;
+    const NodeMaps &maps = GROUP ? mapsg[T.slot] : maps1;
+    const int n0 = d.n[0], n1 = d.n[1], n2 = d.n[2];
+    const int3 zlo = make_int3(T.zlo[0], T.zlo[1], T.zlo[2]);
+    const int3 zhi = make_int3(T.zhi[0], T.zhi[1], T.zhi[2]);
+    const int tcols = T.tcols;
+    const int nplanes = zhi.z - zlo.z;
+    const int64_t rl = r - T.u0, rl1 = min(r1, T.u0 + T.units) - T.u0;  // task-local units
+    const int col = (int)(rl / nplanes);
+    const int zk0 = zlo.z + (int)(rl - (int64_t)col * nplanes);
+    const int zk1 = zlo.z + (int)min((int64_t)nplanes, rl1 - (int64_t)col * nplanes);
+    r = T.u0 + (int64_t)col * nplanes + (zk1 - zlo.z);
+    const int gz_lo = -(int)d.lo[2], gz_hi = d.N[2] - (int)d.lo[2];
     // this segment's zones: local [zi0, zi0+32) x [zj0, zj0+8) x [zk0, zk1) inside [zlo, zhi):
     // the owned zones plus the ghost ring where a neighbour domain exists (ghost zones beyond
     // the physical boundary do not exist; their P stays 0)
@@ -266,41 +279,80 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + ZOFF_RED);
 }
 
+
+// Tiling of one domain's zone stage: ghost ring only on sides with a neighbouring domain.
+ZoneTask zone_task(const DomView &d, int slot) {
+  ZoneTask T = {};
+  T.slot = slot;
+  for (int a = 0; a < 3; ++a) {
+    T.zlo[a] = d.lo[a] > 0 ? -1 : 0;
+    T.zhi[a] = d.lo[a] + d.n[a] < d.N[a] ? d.n[a] + 1 : d.n[a];
+  }
+  T.tcols = (T.zhi[0] - T.zlo[0] + ZBX - 1) / ZBX;
+  const int ty = (T.zhi[1] - T.zlo[1] + ZBY - 1) / ZBY;
+  T.units = (int64_t)T.tcols * ty * (T.zhi[2] - T.zlo[2]);
+  T.u0 = 0;
+  return T;
+}
+
+int zone_slots() {
+  static int slots = 0;
+  if (!slots) {
+    int dev = 0, sms = 0, per_sm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    for (auto k : {k_zone_stage<false>, k_zone_stage<true>})
+      cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ZBYTES);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_zone_stage<false>, ZBX * ZBY,
+                                                  ZBYTES);
+    slots = sms * std::max(per_sm, 1);
+  }
+  return slots;
+}
+
 }  // namespace
 
 int zone_box_y() { return ZNY; }
 
 void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                        cudaStream_t s) {
-  static int slots = 0;
-  if (!slots) {
-    int dev = 0, sms = 0, per_sm = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaFuncSetAttribute(k_zone_stage, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ZBYTES);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_zone_stage, ZBX * ZBY, ZBYTES);
-    slots = sms * std::max(per_sm, 1);
-  }
-  int lo[3], hi[3];
-  for (int a = 0; a < 3; ++a) {  // ghost ring only on sides with a neighbouring domain
-    lo[a] = d.lo[a] > 0 ? -1 : 0;
-    hi[a] = d.lo[a] + d.n[a] < d.N[a] ? d.n[a] + 1 : d.n[a];
-  }
-  const int nz_x = hi[0] - lo[0], nz_y = hi[1] - lo[1], nz_z = hi[2] - lo[2];
-  const int tx = (nz_x + ZBX - 1) / ZBX, ty = (nz_y + ZBY - 1) / ZBY;
+  const int slots = zone_slots();
+  const ZoneTask T = zone_task(d, 0);
   // Default: the persistent linearised split (measured 67 vs 70 us for the best chunking at
   // 128^3).  HYDRO_KZ_ZONE=k: the chunked schedule with k planes per CTA (A/B measurement).
   static const int kz_env = getenv("HYDRO_KZ_ZONE") ? atoi(getenv("HYDRO_KZ_ZONE")) : 0;
-  const int64_t units = (int64_t)tx * ty * nz_z;
+  const int nz = T.zhi[2] - T.zlo[2];
   int G, kz = 0;
   if (kz_env > 0) {
-    kz = std::min(kz_env, nz_z);
-    G = tx * ty * ((nz_z + kz - 1) / kz);
+    kz = std::min(kz_env, nz);
+    G = (int)(T.units / nz) * ((nz + kz - 1) / kz);
   } else {
-    G = (int)std::min<int64_t>(slots, units);
+    G = (int)std::min<int64_t>(slots, T.units);
   }
-  launch_pdl(k_zone_stage, dim3(G), dim3(ZBX * ZBY), ZBYTES, s, maps, d, ph, st, tx, kz, lo[0],
-             lo[1], lo[2], hi[0], hi[1], hi[2]);
+  launch_pdl(k_zone_stage<false>, dim3(G), dim3(ZBX * ZBY), ZBYTES, s, maps, d, T,
+             (const DomView *)nullptr, (const NodeMaps *)nullptr, (const ZoneTask *)nullptr,
+             T.units, kz, ph, st);
+}
+
+void zone_group_tasks(const DomView *views_host, int n, ZoneTask *out, int64_t *Wtot) {
+  int64_t u = 0;
+  for (int i = 0; i < n; ++i) {
+    out[i] = zone_task(views_host[i], i);
+    out[i].u0 = u;
+    u += out[i].units;
+  }
+  *Wtot = u;
+}
+
+void launch_zone_stage_group(const DomView *views_dev, const NodeMaps *maps_dev,
+                             const ZoneTask *tasks_dev, int64_t Wtot, const Phys &ph,
+                             DevState *st, cudaStream_t s) {
+  const int G = (int)std::min<int64_t>(zone_slots(), Wtot);
+  DomView d0 = {};
+  NodeMaps m0 = {};
+  ZoneTask t0 = {};
+  launch_pdl(k_zone_stage<true>, dim3(G), dim3(ZBX * ZBY), ZBYTES, s, m0, d0, t0, views_dev,
+             maps_dev, tasks_dev, Wtot, 0, ph, st);
 }
 
 }  // namespace hydro

@@ -40,6 +40,15 @@ struct HaloCopy {  // one chunk of an intra-GPU ghost slab copy (global boxes, h
 };
 constexpr int HALO_CHUNK = 2048;  // elements per chunk (one CTA of 256 threads)
 
+// Zone-stage work of one domain (kernel_zone.cu): zone box [zlo, zhi) in local indices (the ghost
+// ring where a neighbour exists), tcols x-tiles, `units` = columns x planes, u0 = first unit in
+// the concatenation over the GPU's domains (grouped launch).
+struct ZoneTask {
+  int32_t slot, tcols;
+  int32_t zlo[3], zhi[3];
+  int64_t u0, units;
+};
+
 // Initialisation.
 void launch_init_nodes(const DomView &d, const double origin[3], const double extent[3],
                        cudaStream_t s);
@@ -78,6 +87,24 @@ size_t fused_smem_bytes();
 int fused_box_y();
 
 // Two-kernel cycle (default path): zone stage (P, dt) then node/energy stage.
+// Node/energy-stage work of one domain in a grouped launch (kernel_cycle.cu): x-tiles, columns,
+// z-chunk length and the first CTA of the domain in the concatenated grid.
+struct NodeTask {
+  int32_t slot, tcols, ncols, kz, cta0;
+};
+// Fills out[n] (chunk length shared by all domains); returns the total CTA count.
+int node_group_tasks(const DomView *views_host, int n, NodeTask *out);
+void launch_node_energy_group(const NodeTask *tasks_dev, int ntasks, int nctas,
+                              const DomView *views_dev, const NodeMaps *maps_dev, const Phys &ph,
+                              DevState *st, cudaStream_t s);
+
+// Grouped zone stage over all local domains (one persistent launch): tasks from
+// zone_group_tasks (host), copied to the device by the caller; views_dev / maps_dev indexed by
+// ZoneTask::slot.
+void zone_group_tasks(const DomView *views_host, int n, ZoneTask *out, int64_t *Wtot);
+void launch_zone_stage_group(const DomView *views_dev, const NodeMaps *maps_dev,
+                             const ZoneTask *tasks_dev, int64_t Wtot, const Phys &ph,
+                             DevState *st, cudaStream_t s);
 void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                        cudaStream_t s);
 void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,

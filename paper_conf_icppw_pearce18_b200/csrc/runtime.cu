@@ -49,6 +49,14 @@ struct hydro_ctx {
   DevState *st = nullptr;
   DomView *views_dev[2] = {nullptr, nullptr};
   HaloCopy *local_pairs_dev = nullptr;
+  // grouped zone stage over all local domains (kernel_zone.cu launch_zone_stage_group)
+  NodeMaps *zmaps_dev[2] = {nullptr, nullptr};
+  ZoneTask *ztasks_dev = nullptr;
+  int64_t zunits = 0;
+  bool group = false;
+  NodeMaps *nmaps_dev[2] = {nullptr, nullptr};  // grouped node/energy stage
+  NodeTask *ntasks_dev = nullptr;
+  int nctas = 0;
   int n_local_pairs = 0;
   cudaGraphExec_t graph[2] = {nullptr, nullptr};
   int parity = 0;
@@ -299,6 +307,30 @@ void launch_node_stage(hydro_ctx *h, LocalDom &D, int par, cudaStream_t s) {
   launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
 }
 
+void launch_zone_stages(hydro_ctx *h, int par, cudaStream_t s) {
+  if (h->group)
+    launch_zone_stage_group(h->views_dev[par], h->zmaps_dev[par], h->ztasks_dev, h->zunits,
+                            h->ph, h->st, s);
+  else
+    for (LocalDom &D : h->doms) launch_zone_stage(D.view[par], D.zmaps[par], h->ph, h->st, s);
+}
+
+// The grouped node/energy launch is measured slower on large domains (512^3 in 8 domains: 695
+// vs 614 us per domain; uneven 448^3: equal), so per-domain launches stay the default;
+// HYDRO_GROUP_NODE=1 selects it (A/B).
+bool group_node() {
+  static const int on = getenv("HYDRO_GROUP_NODE") ? atoi(getenv("HYDRO_GROUP_NODE")) : 0;
+  return on != 0;
+}
+
+void launch_node_stages(hydro_ctx *h, int par, cudaStream_t s) {
+  if (h->group && group_node())
+    launch_node_energy_group(h->ntasks_dev, (int)h->doms.size(), h->nctas, h->views_dev[par],
+                             h->nmaps_dev[par], h->ph, h->st, s);
+  else
+    for (LocalDom &D : h->doms) launch_node_stage(h, D, par, s);
+}
+
 // Enqueue one cycle on stream s reading parity `par`.
 int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
   for (LocalDom &D : h->doms) {
@@ -320,12 +352,12 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
       if (rc) return set_err(h, rc, "dt allreduce failed");
     }
   } else {
-    for (LocalDom &D : h->doms) launch_zone_stage(D.view[par], D.zmaps[par], h->ph, h->st, s);
+    launch_zone_stages(h, par, s);
     if (h->comm) {
       int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
     }
-    for (LocalDom &D : h->doms) launch_node_stage(h, D, par, s);
+    launch_node_stages(h, par, s);
   }
   launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
   if (h->comm) {
@@ -519,6 +551,37 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
            if (!vv.empty())
              CK(cudaMemcpyAsync(h->views_dev[par], vv.data(), sizeof(DomView) * vv.size(),
                                 cudaMemcpyHostToDevice, h->stream));
+         }
+         // several domains on this GPU: one grouped zone-stage launch covers them all
+         // (HYDRO_NO_GROUP=1: one launch per domain, for A/B)
+         h->group = h->doms.size() > 1 && !h->split && !h->one_kernel &&
+                    !(getenv("HYDRO_NO_GROUP") && atoi(getenv("HYDRO_NO_GROUP")));
+         if (h->group) {
+           std::vector<DomView> vv;
+           for (LocalDom &D : h->doms) vv.push_back(D.view[0]);
+           std::vector<ZoneTask> tasks(vv.size());
+           zone_group_tasks(vv.data(), (int)vv.size(), tasks.data(), &h->zunits);
+           CK(cudaMalloc(&h->ztasks_dev, sizeof(ZoneTask) * tasks.size()));
+           CK(cudaMemcpy(h->ztasks_dev, tasks.data(), sizeof(ZoneTask) * tasks.size(),
+                         cudaMemcpyHostToDevice));
+           for (int par = 0; par < 2; ++par) {
+             std::vector<NodeMaps> mm, nm;
+             for (LocalDom &D : h->doms) {
+               mm.push_back(D.zmaps[par]);
+               nm.push_back(D.maps[par]);
+             }
+             CK(cudaMalloc(&h->zmaps_dev[par], sizeof(NodeMaps) * mm.size()));
+             CK(cudaMemcpy(h->zmaps_dev[par], mm.data(), sizeof(NodeMaps) * mm.size(),
+                           cudaMemcpyHostToDevice));
+             CK(cudaMalloc(&h->nmaps_dev[par], sizeof(NodeMaps) * nm.size()));
+             CK(cudaMemcpy(h->nmaps_dev[par], nm.data(), sizeof(NodeMaps) * nm.size(),
+                           cudaMemcpyHostToDevice));
+           }
+           std::vector<NodeTask> nt(vv.size());
+           h->nctas = node_group_tasks(vv.data(), (int)vv.size(), nt.data());
+           CK(cudaMalloc(&h->ntasks_dev, sizeof(NodeTask) * nt.size()));
+           CK(cudaMemcpy(h->ntasks_dev, nt.data(), sizeof(NodeTask) * nt.size(),
+                         cudaMemcpyHostToDevice));
          }
          std::vector<HaloCopy> lp;
          std::vector<HaloPair> remote;
@@ -853,7 +916,8 @@ int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, 
 int hydro_kernels_per_cycle(const hydro_ctx *h) {
   if (!h) return HYDRO_EINVAL;
   const int nd = (int)h->doms.size();
-  int k = (h->split ? 3 : (h->one_kernel ? 1 : 2)) * nd;  // cycle kernels
+  int k = h->group ? 1 + (group_node() ? 1 : nd)
+                   : (h->split ? 3 : (h->one_kernel ? 1 : 2)) * nd;  // cycle kernels
   if (h->n_local_pairs > 0) k += 1;  // intra-GPU halo copy
   if (!fold_finalize(h)) k += 1;     // finalize
   if (h->comm) k += comm_kernels_per_cycle(h->comm);
@@ -884,10 +948,10 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
       for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
       if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
     } else {
-      for (LocalDom &D : h->doms) launch_zone_stage(D.view[par], D.zmaps[par], h->ph, h->st, s);
+      launch_zone_stages(h, par, s);
       if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
       CK(cudaEventRecord(ev[4], s));
-      for (LocalDom &D : h->doms) launch_node_stage(h, D, par, s);
+      launch_node_stages(h, par, s);
     }
     CK(cudaEventRecord(ev[1], s));
     launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
@@ -934,6 +998,10 @@ int hydro_destroy(hydro_ctx *h) {
   for (int p = 0; p < 2; ++p) {
     if (h->graph[p]) cudaGraphExecDestroy(h->graph[p]);
     if (h->views_dev[p]) cudaFree(h->views_dev[p]);
+    if (h->zmaps_dev[p]) cudaFree(h->zmaps_dev[p]);
+    if (h->nmaps_dev[p]) cudaFree(h->nmaps_dev[p]);
+    if (p == 0 && h->ntasks_dev) cudaFree(h->ntasks_dev);
+    if (p == 0 && h->ztasks_dev) cudaFree(h->ztasks_dev);
   }
   if (h->comm) comm_destroy(h->comm);
   if (h->peer) peer_destroy(h->peer);
