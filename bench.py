@@ -240,6 +240,9 @@ def main():
     ap.add_argument("--transport", default="peer", choices=["peer", "nccl"],
                     help="N>1 halo/dt transport: CUDA IPC peer stores (tested with 2 ranks on one "
                          "GPU) or NCCL send/recv + allreduce")
+    ap.add_argument("--hg", type=float, default=0.0,
+                    help="viscous hourglass coefficient (SURVEY f1, reading R17); > 0 runs the "
+                         "split kernels")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-cycles", type=int, default=100)
     args = ap.parse_args()
@@ -264,8 +267,10 @@ def main():
     from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig
 
     kw, scaling, desc = workload(args.config, ngpu)
+    if args.hg > 0.0:
+        args.path = "split"  # the library runs the split kernels whenever hg_coef > 0
     cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, path=args.path,
-                      transport=args.transport, **kw)
+                      transport=args.transport, hg_coef=args.hg, **kw)
     hyd = Hydro(cfg)
     n = kw["n"]
     zones = n[0] * n[1] * n[2]
@@ -389,7 +394,7 @@ def main():
             "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
             "config": {"workload": desc, "mesh": list(n), "domains": list(cfg.ndom),
-                       "zones": zones, "path": args.path,
+                       "zones": zones, "path": args.path, "hg_coef": args.hg,
                        "l2": "state > 126 MB L2 (inputs larger than L2; no flush)"
                        if zones * 120 > 126e6 else "state fits L2",
                        "parallelism": f"dp{ngpu} (spatial domains)",

@@ -27,14 +27,19 @@ for vals in rows[2:]:
             return float(d[k].replace(",", ""))
         except (KeyError, ValueError):
             return float("nan")
-    rd, wr = f("dram__bytes_read.sum"), f("dram__bytes_write.sum")
-    unit = 1e6  # ncu reports Mbyte
+    scale = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "B": 1.0, "KB": 1e3,
+             "MB": 1e6, "GB": 1e9}
+    units = dict(zip(hdr, rows[1]))
+    rd = f("dram__bytes_read.sum") * scale[units["dram__bytes_read.sum"]]
+    wr = f("dram__bytes_write.sum") * scale[units["dram__bytes_write.sum"]]
+    unit = 1.0  # bytes (ncu scales each metric's unit; the units row says which)
     regex = "k_zone_stage" if key == "k_zone_stage" else "k_cycle"
     fp = subprocess.run([sys.executable, "tools/ncu_fp64_count.py", rep, regex],
                         capture_output=True, text=True).stdout.split()
     fp64 = float(fp[1]) if len(fp) > 1 else float("nan")
     out[key] = {
-        "duration_us": f("gpu__time_duration.sum"),
+        "duration_us": f("gpu__time_duration.sum") * {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0,
+                                                      "us": 1.0, "msecond": 1e3, "ms": 1e3}[units["gpu__time_duration.sum"]],
         "dram_bytes": (rd + wr) * unit, "dram_read_bytes": rd * unit, "dram_write_bytes": wr * unit,
         "dram_bytes_per_zone": (rd + wr) * unit / zones,
         "fp64_inst": fp64, "fp64_inst_per_zone": fp64 / zones,
