@@ -459,6 +459,9 @@ class Hydro:
         if rc != 0:
             raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
 
+    def _to_device(self, t):
+        return t.to(f"cuda:{self.cfg.device}")
+
     def set_clock(self, t: float, dt: float, cycle: int):
         rc = self._L.hydro_set_clock(self._h, float(t), float(dt), int(cycle))
         if rc != 0:
@@ -515,7 +518,7 @@ class Hydro:
                 for r in dist.batch_isend_irecv(ops):
                     r.wait()
             for d, t in recvd.items():
-                bufs[d] = t.to(f"cuda:{cfg.device}")
+                bufs[d] = self._to_device(t)
         self.close()
         self._create(dataclasses.replace(cfg, dom_to_rank=new_map, rank_weight=None))
         for d in range(len(new_map)):

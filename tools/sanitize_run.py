@@ -5,9 +5,13 @@ from paper_conf_icppw_pearce18_b200.inputs import jittered_state
 
 n = (40, 30, 20)
 cuts = [[0, 17, 40], [0, 12, 30], [0, 20]]
-for path in sys.argv[1:] or ["two", "one", "split"]:
+for path in sys.argv[1:] or ["two", "one", "split", "hg", "single"]:
     kw = dict(n=n, ndom=(2, 2, 1), cuts=cuts, init="user", user=jittered_state(n, 3), path=path,
               graph=False)
+    if path == "hg":  # hourglass control (split kernels)
+        kw.update(path="split", hg_coef=0.03)
+    if path == "single":  # one domain: the persistent zone stage without grouping
+        kw.update(path="two", ndom=(1, 1, 1), cuts=None)
     with Hydro(HydroConfig(**kw)) as h:
         r = h.step(3)
         f = h.fields(["e", "rho"])
