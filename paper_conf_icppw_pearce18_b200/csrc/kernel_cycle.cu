@@ -55,9 +55,13 @@ struct CTile {
   static constexpr int OFF_RAW = 0;                 // [3 slots][NF fields][RS] (TMA)
   static constexpr int OFF_ZR = OFF_RAW + 3 * NF * RS;  // [3 slots][3 fields][ZRS] m, e, P (TMA)
   static constexpr int OFF_XP = OFF_ZR + 9 * ZRS;   // [2 planes][3][RS] half-step positions
-  static constexpr int OFF_G = OFF_XP + 6 * RS;     // [3 vectors][3][ZS] g_x, g_y, g_z
+  // PAD doubles after XP and UH: the padding lanes (t >= NZT) run the unconditional corner and
+  // u_half neighbour loads up to PX + 1 entries past their array; the pad keeps those dead reads
+  // inside dead memory instead of the next array (racecheck-clean)
+  static constexpr int PAD = 64;
+  static constexpr int OFF_G = OFF_XP + 6 * RS + PAD;  // [3 vectors][3][ZS] g_x, g_y, g_z
   static constexpr int OFF_UH = OFF_G + 9 * ZS;     // [3][ZS] u_half of node plane p
-  static constexpr int OFF_P = OFF_UH + 3 * ZS;     // [ZS] P of zone plane p (FUSED)
+  static constexpr int OFF_P = OFF_UH + 3 * ZS + PAD;  // [ZS] P of zone plane p (FUSED)
   static constexpr int OFF_PS = OFF_P + ZS;         // [2][ZS] psi of x-low, y-low faces
   static constexpr int OFF_RED = OFF_PS + 2 * ZS;   // [32] block dt reduction
   static constexpr int OFF_BAR = OFF_RED + 32;      // 3 TMA mbarriers + 3 phase mbarriers
