@@ -339,6 +339,10 @@ def main():
         if flops:
             alu = flops / (kms * 1e-3)
             r.update({"fp64_inst_per_s": alu, "fp64_frac": alu / fp64_peak()})
+        c = KC.get(name)
+        if c:  # the same kernel under ncu at 128^3 (profiles/kernel_counters.json)
+            r["ncu_128"] = {k: c.get(k) for k in ("fp64_pipe_pct", "smem_wavefronts_pct",
+                                                  "issue_active", "dram_bytes_per_zone")}
         rows.append(r)
     dom = max(rows, key=lambda r: r["ms"])
     alu_bound = dom.get("fp64_frac", 0.0) > dom["hbm_frac"]

@@ -48,6 +48,10 @@ for vals in rows[2:]:
         "warps_active": f("sm__warps_active.avg.per_cycle_active"),
         "registers": f("launch__registers_per_thread"),
         "warp_inst": f("smsp__inst_executed.sum"),
+        # shared-memory data-pipe wavefronts (the node stage's binding resource)
+        "smem_wavefronts": f("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum"),
+        "smem_wavefronts_pct": f("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum"
+                                 ".pct_of_peak_sustained_elapsed"),
     }
 json.dump({"report": rep, "zones": zones, "kernels": out}, sys.stdout, indent=1)
 print()
