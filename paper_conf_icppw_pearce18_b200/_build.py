@@ -60,5 +60,20 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+def build_c_example() -> str:
+    """examples/sedov.c against include/hydro.h only (plain C99, no Python): build/sedov_c."""
+    out_dir = os.path.join(ROOT, "build")
+    os.makedirs(out_dir, exist_ok=True)
+    exe = os.path.join(out_dir, "sedov_c")
+    cmd = ["gcc", "-O2", "-std=c99", "-Wall", "-Werror", "-I", os.path.join(ROOT, "include"),
+           os.path.join(ROOT, "examples", "sedov.c"), "-L", HERE, "-l:libhydro_b200.so",
+           "-Wl,-rpath," + HERE, "-lm", "-o", exe]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        sys.stderr.write(r.stdout + r.stderr)
+        raise RuntimeError("C example build failed")
+    return exe
+
+
 if __name__ == "__main__":
     print(build(force=True, verbose="-v" in sys.argv))

@@ -48,6 +48,9 @@ struct CTile {
   static constexpr int ZN = ZBX * ZBY;
   static constexpr int ZRS = (ZN + 15) / 16 * 16;
   // shared memory, in doubles; SoA everywhere so a warp's LDS.64 is conflict-free
+#ifndef HYDRO_ARRIVE_ALL
+#define HYDRO_ARRIVE_ALL 0
+#endif
 #ifndef HYDRO_MN8_TMA
 #define HYDRO_MN8_TMA 1
 #endif
@@ -126,7 +129,8 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   if (!halted && t == 0) {
     if (smem_u32(sm) & 127u) __trap();  // TMA destinations must be 128-byte aligned
     for (int s = 0; s < 3; ++s) mbar_init(&bar[s], 1);
-    for (int s = 3; s < 6; ++s) mbar_init(&bar[s], T::NTHR / 32);  // one arrival per warp
+    for (int s = 3; s < 6; ++s)  // one arrival per warp (HYDRO_ARRIVE_ALL: per thread)
+      mbar_init(&bar[s], HYDRO_ARRIVE_ALL ? T::NTHR : T::NTHR / 32);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
@@ -284,8 +288,12 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   // per plane, so plane p waits on parity (p - q0) & 1.  The fused kernel uses __syncthreads.
   enum { B_G = 3, B_U = 4, B_P = 5 };
   auto arrive = [&](int b) {
-    __syncwarp();
-    if ((t & 31) == 0) mbar_arrive(&bar[b]);
+    if (HYDRO_ARRIVE_ALL) {
+      mbar_arrive(&bar[b]);
+    } else {
+      __syncwarp();
+      if ((t & 31) == 0) mbar_arrive(&bar[b]);
+    }
   };
   auto await = [&](int b, int p) { mbar_wait(&bar[b], (pbase + (uint32_t)(p - q0)) & 1u); };
   auto energy2 = [&](int zp, const Carry &c) {  // E2 of zone plane zp from its carry set
