@@ -48,8 +48,13 @@ struct CTile {
   static constexpr int ZN = ZBX * ZBY;
   static constexpr int ZRS = (ZN + 15) / 16 * 16;
   // shared memory, in doubles; SoA everywhere so a warp's LDS.64 is conflict-free
+// Phase-barrier arrivals: every thread arrives (release) on its own.  The warp-elected variant
+// (__syncwarp, then lane 0 arrives; HYDRO_ARRIVE_ALL=0) is correct under the PTX memory model
+// (bar.warp.sync orders the lanes' stores before lane 0's cumulative release) and measured
+// equally fast, but compute-sanitizer racecheck does not follow that chain and reports every
+// phase as a hazard; per-thread arrivals are racecheck-clean at the same speed (94.2 vs 94.3 us).
 #ifndef HYDRO_ARRIVE_ALL
-#define HYDRO_ARRIVE_ALL 0
+#define HYDRO_ARRIVE_ALL 1
 #endif
 #ifndef HYDRO_MN8_TMA
 #define HYDRO_MN8_TMA 1
