@@ -25,7 +25,10 @@ namespace {
 #ifndef HYDRO_ZONE_MINB
 #define HYDRO_ZONE_MINB 2
 #endif
-constexpr int ZBX = 32, ZBY = 8;                       // zones per block (x, y)
+#ifndef HYDRO_ZONE_BY
+#define HYDRO_ZONE_BY 8
+#endif
+constexpr int ZBX = 32, ZBY = HYDRO_ZONE_BY;           // zones per block (x, y)
 constexpr int ZNX = ZONE_BOX_X, ZNY = ZBY + 1;         // TMA node box (x padded to 16 B)
 constexpr int ZNN = ZNX * ZNY;
 constexpr int ZRS = (ZNN + 15) / 16 * 16;              // stride of one node array (128 B)
