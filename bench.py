@@ -243,6 +243,9 @@ def main():
     ap.add_argument("--hg", type=float, default=0.0,
                     help="viscous hourglass coefficient (SURVEY f1, reading R17); > 0 runs the "
                          "split kernels")
+    ap.add_argument("--halo", default="kernel", choices=["kernel", "fused"],
+                    help="ghost-slab exchange: from the node/energy stage's epilogue (fused) or "
+                         "separate copy / peer-push kernels after it")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-cycles", type=int, default=100)
     args = ap.parse_args()
@@ -270,7 +273,7 @@ def main():
     if args.hg > 0.0:
         args.path = "split"  # the library runs the split kernels whenever hg_coef > 0
     cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, path=args.path,
-                      transport=args.transport, hg_coef=args.hg, **kw)
+                      transport=args.transport, hg_coef=args.hg, halo=args.halo, **kw)
     hyd = Hydro(cfg)
     n = kw["n"]
     zones = n[0] * n[1] * n[2]
@@ -398,7 +401,7 @@ def main():
             "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
             "config": {"workload": desc, "mesh": list(n), "domains": list(cfg.ndom),
-                       "zones": zones, "path": args.path, "hg_coef": args.hg,
+                       "zones": zones, "path": args.path, "hg_coef": args.hg, "halo": args.halo,
                        "l2": "state > 126 MB L2 (inputs larger than L2; no flush)"
                        if zones * 120 > 126e6 else "state fits L2",
                        "parallelism": f"dp{ngpu} (spatial domains)",

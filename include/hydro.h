@@ -71,6 +71,11 @@ enum {
 #define HYDRO_FLAG_PEER (1ull << 3)       /* nranks > 1: exchange halos and reduce dt through peer
                                              memory (CUDA IPC; ranks may share a GPU) instead of
                                              NCCL; needs hydro_peer_export/import after create */
+#define HYDRO_FLAG_HALO_FUSED (1ull << 4) /* default path: the node/energy stage stores the ghost
+                                             slabs into the neighbours (intra-GPU and peer) from
+                                             its own epilogue instead of the separate copy / push
+                                             kernels after it (correct, measured
+                                             slower on B200, so opt-in) */
 
 typedef struct {
   int32_t abi_version;          /* must be HYDRO_ABI_VERSION */

@@ -80,6 +80,7 @@ struct CTile {
   static_assert((ZBX * 8) % 16 == 0, "TMA zone box rows must be 16-byte multiples");
   static_assert(ZRS >= ZS - 32 && ZN <= ZS, "zone tile fits the thread tile");
   static_assert(BYTES <= 227 * 1024, "shared memory");
+  static_assert(9 * ZS * sizeof(double) >= (64 * 8 + 2) * sizeof(int), "fused-halo table");
 };
 
 // GROUP: one chunked launch over all domains of this GPU; CTA b belongs to the NodeTask whose
@@ -88,7 +89,8 @@ template <int TX, int TY, bool FUSED, bool GROUP>
 __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     k_cycle(const __grid_constant__ NodeMaps maps1, const __grid_constant__ DomView d1, Phys ph,
             DevState *st, int tcols1, int ncols1, int sched_kz1, int fold_finalize,
-            const NodeTask *tasks, int ntasks, const DomView *views, const NodeMaps *mapsg) {
+            const NodeTask *tasks, int ntasks, const DomView *views, const NodeMaps *mapsg,
+            const PushSlab *push1, int npush1) {
   using T = CTile<TX, TY>;
   // dynamic shared memory only (no static __shared__), so the window is 1024-byte aligned
   extern __shared__ __align__(1024) double sm[];
@@ -108,6 +110,8 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   const int tcols = GROUP ? tasks[task_i].tcols : tcols1;
   const int sched_kz = GROUP ? tasks[task_i].kz : sched_kz1;
   const int bid = GROUP ? (int)blockIdx.x - tasks[task_i].cta0 : (int)blockIdx.x;
+  const PushSlab *push = GROUP ? push1 + tasks[task_i].push0 : push1;
+  const int npush = GROUP ? tasks[task_i].npush : npush1;
   const int t = threadIdx.x;
   const int n0 = d.n[0], n1 = d.n[1], n2 = d.n[2];
   // lanes: zone/node (tx, ty) for tx < TXT; tx == TXT forms the box's last node column; the
@@ -140,6 +144,128 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   }
   __syncthreads();
   double dt2min = INFINITY;
+
+  // Fused halo: after a column segment, the CTA stores the part of every
+  // neighbour's ghost slab that it has just written (nodes of planes [k0, k1), plus n2 on the
+  // last chunk; zones of planes [k0, k1)) into the neighbour's next-parity arrays, reading the
+  // values back from its own freshly written (L2-resident) output.  Replaces the separate
+  // intra-GPU copy / peer push kernel: the exchange overlaps the other CTAs' compute.  Warp 0
+  // clips the (<= 32) slabs against the segment in parallel, one lane per slab, and scans the
+  // item counts into a table in the (now idle) g-vector smem; then every (slab, kind, element)
+  // item is one independent load/store for some thread.
+  auto push_halo = [&](int i0, int j0, int k0, int k1) {
+    int *tab = reinterpret_cast<int *>(sm + T::OFF_G);  // [64 items][8]: end, lo x3, ext x2, slab, kind
+    if (t < 32) {
+      // this segment's output: nodes [i0, wn1) x [j0, wn1) x [k0, wn1), zones [.., wz1); the last
+      // tile in x / y also writes the domain's last node (F_NWR), the last chunk node plane n2
+      const int wn1[3] = {n0 <= i0 + TX ? n0 + 1 : i0 + TX, n1 <= j0 + TY ? n1 + 1 : j0 + TY,
+                          k1 == n2 ? n2 + 1 : k1};
+      const int wz1[3] = {min(i0 + TX, n0), min(j0 + TY, n1), k1};
+      const int w0[3] = {i0, j0, k0};
+      int cnt[2] = {0, 0}, lo[2][3] = {}, ext[2][3] = {}, rem = 0;
+      if (t < npush) {
+        const PushSlab &S = push[t];
+        rem = S.remote;
+#pragma unroll
+        for (int c = 0; c < 2; ++c) {
+          int n = 1;
+#pragma unroll
+          for (int a = 0; a < 3; ++a) {
+            lo[c][a] = max(c ? S.zlo[a] : S.nlo[a], w0[a]);
+            ext[c][a] = min(c ? S.zhi[a] : S.nhi[a], c ? wz1[a] : wn1[a]) - lo[c][a];
+            n = ext[c][a] > 0 ? n * ext[c][a] : 0;
+          }
+          cnt[c] = n;
+        }
+      }
+      int incl = cnt[0] + cnt[1];  // inclusive warp scan of the per-slab item counts
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(0xffffffffu, incl, o);
+        if (t >= o) incl += v;
+      }
+      const int excl = incl - cnt[0] - cnt[1];
+#pragma unroll
+      for (int c = 0; c < 2; ++c) {
+        int *r = tab + (2 * t + c) * 8;
+        r[0] = excl + cnt[0] + (c ? cnt[1] : 0);  // end of the item range
+        r[1] = lo[c][0]; r[2] = lo[c][1]; r[3] = lo[c][2];
+        r[4] = ext[c][0]; r[5] = ext[c][1];
+        r[6] = t; r[7] = c;
+      }
+      const bool any_remote = __any_sync(0xffffffffu, rem && (cnt[0] + cnt[1]) > 0);
+      if (t == 31) {
+        tab[64 * 8] = incl;
+        tab[64 * 8 + 1] = any_remote;
+      }
+    }
+    __syncthreads();
+    const int total = tab[64 * 8];
+    const int nsx = (int)d.nsx, nsxy2 = (int)d.nsxy, zsx = (int)d.zsx, zsxy2 = (int)d.zsxy;
+    // two items per thread in flight: both items' loads, then both items' stores
+    struct Item { int kind, si; int64_t di; const PushSlab *S; };
+    auto locate = [&](int e) {
+      int a = 0, b = 63;  // first item whose end exceeds e
+      while (a < b) {
+        const int m = (a + b) >> 1;
+        if (tab[m * 8] > e) b = m;
+        else a = m + 1;
+      }
+      const int *r = tab + a * 8;
+      const int rem = e - (a ? tab[(a - 1) * 8] : 0);
+      const int i = r[1] + rem % r[4], q = rem / r[4];
+      const int j = r[2] + q % r[5], k = r[3] + q / r[5];
+      Item it;
+      it.kind = r[7];
+      it.S = push + r[6];
+      if (it.kind == 0) {
+        it.si = (k + 1) * nsxy2 + (j + 1) * nsx + (i + 1);
+        it.di = __ldg(&it.S->nbase) + (int64_t)k * __ldg(&it.S->nsxy) +
+                (int64_t)j * __ldg(&it.S->nsx) + i;
+      } else {
+        it.si = (k + 1) * zsxy2 + (j + 1) * zsx + (i + 1);
+        it.di = __ldg(&it.S->zbase) + (int64_t)k * __ldg(&it.S->zsxy) +
+                (int64_t)j * __ldg(&it.S->zsx) + i;
+      }
+      return it;
+    };
+    auto load = [&](const Item &it, double &v0, double &v1, double &v2, double &v3, double &v4,
+                    double &v5) {
+      if (it.kind == 0) {
+        v0 = d.xn[it.si]; v1 = d.yn[it.si]; v2 = d.zn[it.si];
+        v3 = d.un[it.si]; v4 = d.vn[it.si]; v5 = d.wn[it.si];
+      } else {
+        v0 = d.en[it.si];
+      }
+    };
+    auto store = [&](const Item &it, double v0, double v1, double v2, double v3, double v4,
+                     double v5) {
+      const long long *dst = (const long long *)it.S->dst;
+      if (it.kind == 0) {
+        ((double *)__ldg(dst + 0))[it.di] = v0;
+        ((double *)__ldg(dst + 1))[it.di] = v1;
+        ((double *)__ldg(dst + 2))[it.di] = v2;
+        ((double *)__ldg(dst + 3))[it.di] = v3;
+        ((double *)__ldg(dst + 4))[it.di] = v4;
+        ((double *)__ldg(dst + 5))[it.di] = v5;
+      } else {
+        ((double *)__ldg(dst + 6))[it.di] = v0;
+      }
+    };
+    for (int e0 = t; e0 < total; e0 += 2 * T::NTHR) {
+      const bool two = e0 + T::NTHR < total;
+      const Item A = locate(e0);
+      const Item B = locate(two ? e0 + T::NTHR : e0);
+      double a0 = 0, a1 = 0, a2 = 0, a3 = 0, a4 = 0, a5 = 0;
+      double b0 = 0, b1 = 0, b2 = 0, b3 = 0, b4 = 0, b5 = 0;
+      load(A, a0, a1, a2, a3, a4, a5);
+      load(B, b0, b1, b2, b3, b4, b5);
+      store(A, a0, a1, a2, a3, a4, a5);
+      if (two) store(B, b0, b1, b2, b3, b4, b5);
+    }
+    if (total && tab[64 * 8 + 1]) __threadfence_system();  // peer stores before the mailbox flag
+    __syncthreads();  // the table region is the next segment's g-vector array
+  };
   uint32_t ubase = 0;  // TMA planes consumed in earlier segments (ring slot / phase continuity)
   uint32_t pbase = 0;  // plane iterations run in earlier segments (phase-barrier parity)
 
@@ -165,6 +291,10 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
         const int64_t z = d.zid(li, lj, p);
         d.en[z] = d.e[z];
       }
+    }
+    if (!FUSED && npush) {
+      __syncthreads();  // the whole segment's output is written
+      push_halo(i0, j0, k0, k1);
     }
     continue;
   }
@@ -537,6 +667,7 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   ubase += (uint32_t)(k1 + 2 - q0);  // node planes q0 .. k1+1 went through the TMA ring
   pbase += (uint32_t)(k1 + 1 - q0);  // iterations p = q0 .. k1 completed each phase barrier
   __syncthreads();                   // the next segment reuses the rings
+  if (!FUSED && npush) push_halo(i0, j0, k0, k1);
   }
   if (FUSED) block_min_dt_smem(sqrt(dt2min), &st->dtz_acc, sm + T::OFF_RED);
   if (fold_finalize)  // single-domain, single-rank cycle: S9 here instead of a separate launch
@@ -587,7 +718,7 @@ int num_sms() {
 
 template <bool FUSED>
 void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st, int fold,
-            cudaStream_t s) {
+            const PushSlab *push, int npush, cudaStream_t s) {
   using T = CTile<CTX, CTY>;
   set_smem<FUSED>();
   const int sms = num_sms();
@@ -608,7 +739,7 @@ void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st
   }
   launch_pdl(k_cycle<CTX, CTY, FUSED, false>, dim3(G), dim3(T::NTHR), T::BYTES, s, maps, d, ph,
              st, tx, ncols, kz, fold, (const NodeTask *)nullptr, 0, (const DomView *)nullptr,
-             (const NodeMaps *)nullptr);
+             (const NodeMaps *)nullptr, push, npush);
 }
 
 }  // namespace
@@ -621,12 +752,12 @@ int cycle_zone_box_y() { return CTile<CTX, CTY>::ZBY; }
 
 void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                         int fold_finalize, cudaStream_t s) {
-  launch<true>(d, maps, ph, st, fold_finalize, s);
+  launch<true>(d, maps, ph, st, fold_finalize, nullptr, 0, s);
 }
 
 void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                        int fold_finalize, cudaStream_t s) {
-  launch<false>(d, maps, ph, st, fold_finalize, s);
+                        int fold_finalize, const PushSlab *push, int npush, cudaStream_t s) {
+  launch<false>(d, maps, ph, st, fold_finalize, push, npush, s);
 }
 
 int node_group_tasks(const DomView *views_host, int n, NodeTask *out) {
@@ -658,6 +789,8 @@ int node_group_tasks(const DomView *views_host, int n, NodeTask *out) {
     T.ncols = T.tcols * ((d.n[1] + CTY - 1) / CTY);
     T.kz = std::min(best, d.n[2]);
     T.cta0 = cta;
+    T.push0 = 0;
+    T.npush = 0;  // filled by the runtime when the fused halo is on
     cta += T.ncols * ((d.n[2] + T.kz - 1) / T.kz);
   }
   return cta;
@@ -665,13 +798,13 @@ int node_group_tasks(const DomView *views_host, int n, NodeTask *out) {
 
 void launch_node_energy_group(const NodeTask *tasks_dev, int ntasks, int nctas,
                               const DomView *views_dev, const NodeMaps *maps_dev, const Phys &ph,
-                              DevState *st, cudaStream_t s) {
+                              DevState *st, const PushSlab *push, cudaStream_t s) {
   using T = CTile<CTX, CTY>;
   set_smem<false>();
   DomView d0 = {};
   NodeMaps m0 = {};
   launch_pdl(k_cycle<CTX, CTY, false, true>, dim3(nctas), dim3(T::NTHR), T::BYTES, s, m0, d0,
-             ph, st, 0, 0, 0, 0, tasks_dev, ntasks, views_dev, maps_dev);
+             ph, st, 0, 0, 0, 0, tasks_dev, ntasks, views_dev, maps_dev, push, 0);
 }
 
 }  // namespace hydro

@@ -40,6 +40,21 @@ struct HaloCopy {  // one chunk of an intra-GPU ghost slab copy (global boxes, h
 };
 constexpr int HALO_CHUNK = 2048;  // elements per chunk (one CTA of 256 threads)
 
+// One ghost slab a domain stores into a neighbour from the node/energy-stage epilogue (fused
+// halo): the neighbour's ghost nodes / zones that this (source) domain owns, as
+// boxes in SOURCE-local indices, and where they go.  Destination index of the source-local node
+// (i, j, k) = nbase + k nsxy + j nsx + i (zones: zbase, zsxy, zsx); dst = the destination's
+// next-parity x,y,z,u,v,w,e arrays (device pointers on this GPU, or CUDA-IPC mapped peer memory).
+struct PushSlab {
+  int32_t nlo[3], nhi[3];  // node box, half-open
+  int32_t zlo[3], zhi[3];  // zone box, half-open
+  int64_t nbase, zbase;
+  int32_t nsx, nsxy, zsx, zsxy;
+  double *dst[7];
+  int32_t remote;          // destination in another process (system-scope fence after the stores)
+  int32_t pad_;
+};
+
 // Zone-stage work of one domain (kernel_zone.cu): zone box [zlo, zhi) in local indices (the ghost
 // ring where a neighbour exists), tcols x-tiles, `units` = columns x planes, u0 = first unit in
 // the concatenation over the GPU's domains (grouped launch).
@@ -91,12 +106,13 @@ int fused_box_y();
 // z-chunk length and the first CTA of the domain in the concatenated grid.
 struct NodeTask {
   int32_t slot, tcols, ncols, kz, cta0;
+  int32_t push0, npush;  // this domain's PushSlab range (fused halo; npush 0 = none)
 };
 // Fills out[n] (chunk length shared by all domains); returns the total CTA count.
 int node_group_tasks(const DomView *views_host, int n, NodeTask *out);
 void launch_node_energy_group(const NodeTask *tasks_dev, int ntasks, int nctas,
                               const DomView *views_dev, const NodeMaps *maps_dev, const Phys &ph,
-                              DevState *st, cudaStream_t s);
+                              DevState *st, const PushSlab *push, cudaStream_t s);
 
 // Grouped zone stage over all local domains (one persistent launch): tasks from
 // zone_group_tasks (host), copied to the device by the caller; views_dev / maps_dev indexed by
@@ -107,8 +123,10 @@ void launch_zone_stage_group(const DomView *views_dev, const NodeMaps *maps_dev,
                              DevState *st, cudaStream_t s);
 void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                        cudaStream_t s);
+// push/npush: this domain's fused-halo slabs (nullptr/0: none; the caller then exchanges the
+// ghost layer with launch_halo_copy / the transports).
 void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                        int fold_finalize, cudaStream_t s);
+                        int fold_finalize, const PushSlab *push, int npush, cudaStream_t s);
 int zone_box_y();
 int node_box_y();
 int cycle_zone_box_x();  // zone-field TMA box of the cycle kernels

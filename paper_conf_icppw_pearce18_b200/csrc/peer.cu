@@ -110,6 +110,7 @@ struct Peer {
   std::vector<void *> opened;                      // IPC-mapped bases to close
   DomView *remote_dev[2] = {nullptr, nullptr};     // remote destination views per parity
   PeerSlab *slabs_dev = nullptr;
+  std::vector<PushTarget> targets;  // host copy of the slabs (fused halo tables)
   int nslabs = 0;
   int blocks = 1;
   bool ready = false;
@@ -251,6 +252,15 @@ int peer_import(Peer *p, const Layout &L, const std::vector<int32_t> &slot_of_do
     }
     biggest = std::max(biggest, nn);
     slabs.push_back(s);
+    PushTarget pt;
+    pt.src_slot = s.src_slot;
+    pt.remote = 1;
+    for (int a = 0; a < 3; ++a) {
+      pt.nlo[a] = P.nlo[a]; pt.nhi[a] = P.nhi[a]; pt.zlo[a] = P.zlo[a]; pt.zhi[a] = P.zhi[a];
+    }
+    pt.dst[0] = rv[0][s.dst_view];
+    pt.dst[1] = rv[1][s.dst_view];
+    p->targets.push_back(pt);
   }
   p->nslabs = (int)slabs.size();
   p->blocks = (int)std::max<int64_t>(1, std::min<int64_t>(1024, biggest / 1024));
@@ -285,7 +295,11 @@ int peer_exchange(Peer *p, const DomView *local_views_dev, int par, bool halo, D
   return cudaGetLastError() == cudaSuccess ? HYDRO_OK : HYDRO_ECUDA;
 }
 
-int peer_kernels_per_cycle(const Peer *p) { return (p->nslabs ? 1 : 0) + 1; }
+int peer_kernels_per_cycle(const Peer *p, bool halo) { return (halo && p->nslabs ? 1 : 0) + 1; }
+
+void peer_push_targets(const Peer *p, std::vector<PushTarget> *out) {
+  out->insert(out->end(), p->targets.begin(), p->targets.end());
+}
 
 void peer_destroy(Peer *p) {
   if (!p) return;

@@ -12,6 +12,15 @@ namespace hydro {
 
 struct Peer;
 
+// A ghost slab that a local source domain stores into a neighbour (fused halo):
+// global node / zone boxes (half-open) and the destination's views per parity.
+struct PushTarget {
+  int32_t src_slot;
+  int32_t remote;  // destination owned by another process (peer memory)
+  int64_t nlo[3], nhi[3], zlo[3], zhi[3];
+  DomView dst[2];
+};
+
 // Storage helpers shared with the runtime (runtime.cu): a remote domain's arrays are rebuilt
 // from its IPC-mapped base with the same offsets its owner used.
 size_t domain_bytes(const DomainBox &b, bool split);
@@ -31,7 +40,9 @@ bool peer_ready(const Peer *p);
 // and the error bits over all ranks through the mailboxes.
 int peer_exchange(Peer *p, const DomView *local_views_dev, int par, bool halo, DevState *st,
                   cudaStream_t s);
-int peer_kernels_per_cycle(const Peer *p);
+int peer_kernels_per_cycle(const Peer *p, bool halo);
+// The inter-rank slabs this rank pushes (after peer_import), for the fused-halo tables.
+void peer_push_targets(const Peer *p, std::vector<PushTarget> *out);
 void peer_destroy(Peer *p);
 
 }  // namespace hydro

@@ -56,8 +56,14 @@ struct hydro_ctx {
   bool group = false;
   NodeMaps *nmaps_dev[2] = {nullptr, nullptr};  // grouped node/energy stage
   NodeTask *ntasks_dev = nullptr;
+  std::vector<NodeTask> ntasks_host;
   int nctas = 0;
   int n_local_pairs = 0;
+  // fused halo (default two-kernel path): the node/energy stage stores the ghost slabs itself
+  bool fused_halo = false;
+  std::vector<PushTarget> push_targets;     // local and (after peer import) remote slabs
+  PushSlab *push_dev[2] = {nullptr, nullptr};
+  std::vector<int32_t> push_first, push_count;  // per local slot
   cudaGraphExec_t graph[2] = {nullptr, nullptr};
   int parity = 0;
   bool split = false;
@@ -303,8 +309,11 @@ int fold_finalize(const hydro_ctx *h) {
                                                                                            : 0;
 }
 
-void launch_node_stage(hydro_ctx *h, LocalDom &D, int par, cudaStream_t s) {
-  launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
+void launch_node_stage(hydro_ctx *h, LocalDom &D, int par, int slot, cudaStream_t s) {
+  const bool p = h->fused_halo && h->push_dev[par] && h->push_count[slot] > 0;
+  launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h),
+                     p ? h->push_dev[par] + h->push_first[slot] : nullptr,
+                     p ? h->push_count[slot] : 0, s);
 }
 
 void launch_zone_stages(hydro_ctx *h, int par, cudaStream_t s) {
@@ -326,9 +335,68 @@ bool group_node() {
 void launch_node_stages(hydro_ctx *h, int par, cudaStream_t s) {
   if (h->group && group_node())
     launch_node_energy_group(h->ntasks_dev, (int)h->doms.size(), h->nctas, h->views_dev[par],
-                             h->nmaps_dev[par], h->ph, h->st, s);
+                             h->nmaps_dev[par], h->ph, h->st,
+                             h->fused_halo ? h->push_dev[par] : nullptr, s);
   else
-    for (LocalDom &D : h->doms) launch_node_stage(h, D, par, s);
+    for (size_t i = 0; i < h->doms.size(); ++i) launch_node_stage(h, h->doms[i], par, (int)i, s);
+}
+
+// Fused-halo tables: per parity, the PushSlabs of every local source domain,
+// grouped by source slot (push_first / push_count), in source-local boxes.
+int build_push_tables(hydro_ctx *h) {
+  const int ns = (int)h->doms.size();
+  h->push_first.assign(ns, 0);
+  h->push_count.assign(ns, 0);
+  std::vector<PushSlab> tab[2];
+  for (int slot = 0; slot < ns; ++slot) {
+    h->push_first[slot] = (int)tab[0].size();
+    for (const PushTarget &T : h->push_targets) {
+      if (T.src_slot != slot) continue;
+      for (int par = 0; par < 2; ++par) {
+        const DomView &S = h->doms[slot].view[par];
+        const DomView &D = T.dst[par];
+        PushSlab p = {};
+        int o[3];
+        for (int a = 0; a < 3; ++a) {
+          p.nlo[a] = (int32_t)(T.nlo[a] - S.lo[a]);
+          p.nhi[a] = (int32_t)(T.nhi[a] - S.lo[a]);
+          p.zlo[a] = (int32_t)(T.zlo[a] - S.lo[a]);
+          p.zhi[a] = (int32_t)(T.zhi[a] - S.lo[a]);
+          o[a] = (int)(S.lo[a] - D.lo[a]);  // source-local -> destination-local offset
+        }
+        p.nbase = D.nid(o[0], o[1], o[2]);
+        p.zbase = D.zid(o[0], o[1], o[2]);
+        p.nsx = (int32_t)D.nsx;
+        p.nsxy = (int32_t)D.nsxy;
+        p.zsx = (int32_t)D.zsx;
+        p.zsxy = (int32_t)D.zsxy;
+        double *dst[7] = {D.xn, D.yn, D.zn, D.un, D.vn, D.wn, D.en};
+        for (int f = 0; f < 7; ++f) p.dst[f] = dst[f];
+        p.remote = T.remote;
+        tab[par].push_back(p);
+      }
+    }
+    h->push_count[slot] = (int)tab[0].size() - h->push_first[slot];
+    if (h->push_count[slot] > 32)  // one warp lane per slab (kernel_cycle.cu push_halo)
+      return set_err(h, HYDRO_EINVAL, "fused halo: more than 32 ghost slabs from one domain");
+  }
+  for (int par = 0; par < 2; ++par) {
+    if (h->push_dev[par]) CK(cudaFree(h->push_dev[par]));
+    h->push_dev[par] = nullptr;
+    if (tab[par].empty()) continue;
+    CK(cudaMalloc(&h->push_dev[par], sizeof(PushSlab) * tab[par].size()));
+    CK(cudaMemcpy(h->push_dev[par], tab[par].data(), sizeof(PushSlab) * tab[par].size(),
+                  cudaMemcpyHostToDevice));
+  }
+  if (h->group && h->ntasks_dev) {
+    for (int i = 0; i < ns; ++i) {
+      h->ntasks_host[i].push0 = h->push_first[i];
+      h->ntasks_host[i].npush = h->push_count[i];
+    }
+    CK(cudaMemcpy(h->ntasks_dev, h->ntasks_host.data(), sizeof(NodeTask) * ns,
+                  cudaMemcpyHostToDevice));
+  }
+  return HYDRO_OK;
 }
 
 // Enqueue one cycle on stream s reading parity `par`.
@@ -359,13 +427,13 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
     }
     launch_node_stages(h, par, s);
   }
-  launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
+  if (!h->fused_halo) launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
   if (h->comm) {
     int rc = comm_halo(h->comm, par, s);
     if (rc) return set_err(h, rc, "halo exchange failed");
   }
-  if (h->peer) {  // halo push into the peers + dt / error reduction through the mailboxes
-    int rc = peer_exchange(h->peer, h->views_dev[par], par, true, h->st, s);
+  if (h->peer) {  // halo push into the peers (unless fused) + dt / error reduction
+    int rc = peer_exchange(h->peer, h->views_dev[par], par, !h->fused_halo, h->st, s);
     if (rc) return set_err(h, rc, "peer exchange failed");
   }
   if (!fold_finalize(h)) launch_finalize(h->st, h->ph, s);
@@ -577,7 +645,8 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
              CK(cudaMemcpy(h->nmaps_dev[par], nm.data(), sizeof(NodeMaps) * nm.size(),
                            cudaMemcpyHostToDevice));
            }
-           std::vector<NodeTask> nt(vv.size());
+           std::vector<NodeTask> &nt = h->ntasks_host;
+           nt.resize(vv.size());
            h->nctas = node_group_tasks(vv.data(), (int)vv.size(), nt.data());
            CK(cudaMalloc(&h->ntasks_dev, sizeof(NodeTask) * nt.size()));
            CK(cudaMemcpy(h->ntasks_dev, nt.data(), sizeof(NodeTask) * nt.size(),
@@ -589,6 +658,16 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
            const bool dst_local = h->slot_of_dom[P.dst] >= 0;
            const bool src_local = h->slot_of_dom[P.src] >= 0;
            if (dst_local && src_local) {
+             PushTarget pt;
+             pt.src_slot = h->slot_of_dom[P.src];
+             pt.remote = 0;
+             for (int a = 0; a < 3; ++a) {
+               pt.nlo[a] = P.nlo[a]; pt.nhi[a] = P.nhi[a];
+               pt.zlo[a] = P.zlo[a]; pt.zhi[a] = P.zhi[a];
+             }
+             pt.dst[0] = h->doms[h->slot_of_dom[P.dst]].view[0];
+             pt.dst[1] = h->doms[h->slot_of_dom[P.dst]].view[1];
+             h->push_targets.push_back(pt);
              HaloCopy c;
              c.dst = h->slot_of_dom[P.dst];
              c.src = h->slot_of_dom[P.src];
@@ -613,6 +692,11 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
            }
          }
          h->n_local_pairs = (int)lp.size();  // chunk entries
+         h->fused_halo = !h->split && !h->one_kernel && (cfg->flags & HYDRO_FLAG_HALO_FUSED);
+         if (h->fused_halo) {
+           int r = build_push_tables(h);
+           if (r) return r;
+         }
          if (!lp.empty()) {
            CK(cudaMalloc(&h->local_pairs_dev, sizeof(HaloCopy) * lp.size()));
            CK(cudaMemcpyAsync(h->local_pairs_dev, lp.data(), sizeof(HaloCopy) * lp.size(),
@@ -687,6 +771,10 @@ int hydro_peer_import(hydro_ctx *h, const void *all, size_t len_per_rank) {
   CK(cudaSetDevice(h->device));
   int rc = peer_import(h->peer, h->L, h->slot_of_dom, h->split, all, len_per_rank, &h->err);
   if (rc) return rc;
+  if (h->fused_halo) {  // the inter-rank slabs join the node/energy stage's epilogue stores
+    peer_push_targets(h->peer, &h->push_targets);
+    if ((rc = build_push_tables(h)) != HYDRO_OK) return rc;
+  }
   // dt^0 over all ranks (no halo: every rank initialised its ghosts from the global definition)
   rc = peer_exchange(h->peer, h->views_dev[0], 0, false, h->st, h->stream);
   if (rc) return set_err(h, rc, "peer dt^0 exchange failed");
@@ -918,10 +1006,10 @@ int hydro_kernels_per_cycle(const hydro_ctx *h) {
   const int nd = (int)h->doms.size();
   int k = h->group ? 1 + (group_node() ? 1 : nd)
                    : (h->split ? 3 : (h->one_kernel ? 1 : 2)) * nd;  // cycle kernels
-  if (h->n_local_pairs > 0) k += 1;  // intra-GPU halo copy
+  if (h->n_local_pairs > 0 && !h->fused_halo) k += 1;  // intra-GPU halo copy
   if (!fold_finalize(h)) k += 1;     // finalize
   if (h->comm) k += comm_kernels_per_cycle(h->comm);
-  if (h->peer) k += peer_kernels_per_cycle(h->peer);
+  if (h->peer) k += peer_kernels_per_cycle(h->peer, !h->fused_halo);
   return k;
 }
 
@@ -954,9 +1042,10 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
       launch_node_stages(h, par, s);
     }
     CK(cudaEventRecord(ev[1], s));
-    launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
+    if (!h->fused_halo)
+      launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
     if (h->comm && comm_halo(h->comm, par, s)) return HYDRO_ENCCL;
-    if (h->peer && peer_exchange(h->peer, h->views_dev[par], par, true, h->st, s))
+    if (h->peer && peer_exchange(h->peer, h->views_dev[par], par, !h->fused_halo, h->st, s))
       return HYDRO_ECUDA;
     CK(cudaEventRecord(ev[2], s));
     if (!fold_finalize(h)) launch_finalize(h->st, h->ph, s);
@@ -1008,6 +1097,8 @@ int hydro_destroy(hydro_ctx *h) {
   for (LocalDom &D : h->doms)
     if (D.mem) cudaFree(D.mem);
   if (h->local_pairs_dev) cudaFree(h->local_pairs_dev);
+  for (int p = 0; p < 2; ++p)
+    if (h->push_dev[p]) cudaFree(h->push_dev[p]);
   if (h->stage) cudaFree(h->stage);
   if (h->st) cudaFree(h->st);
   if (h->stream) cudaStreamDestroy(h->stream);

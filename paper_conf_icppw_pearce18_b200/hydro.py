@@ -27,6 +27,7 @@ FLAG_NO_GRAPH = 1 << 0
 FLAG_SPLIT = 1 << 1
 FLAG_ONE_KERNEL = 1 << 2
 FLAG_PEER = 1 << 3
+FLAG_HALO_FUSED = 1 << 4
 
 STATUS = {0: "ok", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENCCL", -5: "ETANGLED",
           -6: "ENONFINITE", -7: "EDTMIN", -8: "ESTATE"}
@@ -150,6 +151,9 @@ class HydroConfig:
     graph: bool = True            # CUDA graphs (HYDRO_FLAG_NO_GRAPH when False)
     transport: str = "nccl"       # nranks > 1: "nccl" (NCCL send/recv + allreduce) or "peer"
                                   # (CUDA IPC peer stores + mailbox reduction; ranks may share a GPU)
+    halo: str = "kernel"          # default path: "kernel" (separate copy / peer-push kernels after
+                                  # the node/energy stage) or "fused" (the stage stores the ghost
+                                  # slabs from its own epilogue, HYDRO_FLAG_HALO_FUSED)
     hg_coef: float = 0.0          # viscous hourglass kappa (reading R17); > 0 runs
                                   # the split kernels
 
@@ -199,7 +203,8 @@ def _cfg_struct(cfg: HydroConfig, keep: list, comm_id: Optional[bytes] = None) -
         c.comm_id = C.cast(buf, C.c_void_p)
     c.flags = ((0 if cfg.graph else FLAG_NO_GRAPH) | (FLAG_SPLIT if cfg.path == "split" else 0)
                | (FLAG_ONE_KERNEL if cfg.path == "one" else 0)
-               | (FLAG_PEER if cfg.transport == "peer" else 0))
+               | (FLAG_PEER if cfg.transport == "peer" else 0)
+               | (FLAG_HALO_FUSED if cfg.halo == "fused" else 0))
     return c
 
 

@@ -1,0 +1,85 @@
+"""Fused halo (opt-in HydroConfig.halo="fused"): the node/energy stage stores every
+neighbour's ghost slab from its own epilogue instead of a separate copy kernel after it.  The ghost layer is what PAPER.md
+L548-557 exchanges between neighbouring domains; decomposed runs must equal the undecomposed
+run bitwise (SURVEY §8e ghost contract) and the oracle within the north_star tolerance, with
+either exchange (HydroConfig.halo = "fused" | "kernel")."""
+import numpy as np
+import pytest
+
+import oracle
+from oracle import OracleConfig
+from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig
+from paper_conf_icppw_pearce18_b200.inputs import jittered_state
+from tests.helpers import rel_err
+
+pytestmark = pytest.mark.gpu
+
+FIELDS = ("x", "y", "z", "u", "v", "w", "rho", "e", "p", "q", "c", "vol", "mass")
+
+
+def run(ncycles, **kw):
+    with Hydro(HydroConfig(**kw)) as h:
+        info = h.step(ncycles)
+        f = h.fields()
+    return f, info
+
+
+def _ocfg(kw):
+    keys = ("n", "origin", "extent", "init", "user", "ndom", "cuts", "t_stop")  # no "halo"
+    return OracleConfig(**{k: v for k, v in kw.items() if k in keys})
+
+
+def test_fused_equals_halo_kernels_and_single_domain():
+    # 1-zone-thick domains in y and z: a source's interface node is also its send layer
+    n = (24, 20, 18)
+    cuts = [[0, 5, 13, 24], [0, 1, 20], [0, 9, 10, 18]]
+    kw = dict(n=n, ndom=(3, 2, 3), cuts=cuts, init="user", user=jittered_state(n, 7))
+    ff, i_f = run(25, halo="fused", **kw)
+    fk, i_k = run(25, halo="kernel", **kw)
+    fs, _ = run(25, n=n, init="user", user=kw["user"])
+    assert i_f["status"] == 0 and i_f["dt"] == i_k["dt"]
+    for k in FIELDS:
+        assert np.array_equal(ff[k], fk[k]), k
+        assert np.array_equal(ff[k], fs[k]), k
+
+
+def test_fused_halo_many_tiles_and_z_chunks_against_oracle():
+    # domains several node-stage tiles (32 x 12) wide, tall enough in z for several z-chunks,
+    # so the slabs are split over many CTAs and chunk boundaries
+    n = (70, 50, 90)
+    cuts = [[0, 33, 70], [0, 13, 37, 50], [0, 45, 90]]
+    kw = dict(n=n, ndom=(2, 3, 2), cuts=cuts, init="user", user=jittered_state(n, 12),
+              halo="fused")
+    fg, ig = run(8, **kw)
+    fs, _ = run(8, n=n, init="user", user=kw["user"])
+    for k in FIELDS:
+        assert np.array_equal(fg[k], fs[k]), k
+    fo, io = oracle.run(_ocfg(kw), 8)
+    assert ig["dt"] == pytest.approx(io["dt"], rel=1e-11)
+    for k in FIELDS:
+        assert rel_err(fg[k], fo[k]) <= 1e-11, k
+
+
+def test_fused_halo_no_op_cycles_after_t_stop():
+    # once t_stop is reached the cycles are no-ops that carry the state (and the ghost layer,
+    # through the same epilogue stores) to the next parity
+    n = (16, 16, 16)
+    kw = dict(n=n, ndom=(2, 2, 2), t_stop=0.01, halo="fused")
+    fg, ig = run(400, **kw)
+    fs, is_ = run(400, n=n, t_stop=0.01)
+    assert ig["t"] == pytest.approx(0.01, rel=1e-14) and ig["cycle"] == is_["cycle"]
+    for k in FIELDS:
+        assert np.array_equal(fg[k], fs[k]), k
+    fo, io = oracle.run(_ocfg(kw), 400)
+    assert ig["cycle"] == io["cycle"]
+    for k in FIELDS:
+        assert rel_err(fg[k], fo[k]) <= 1e-10, k
+
+
+def test_kernels_per_cycle_counts_the_fused_exchange():
+    kw = dict(n=(16, 16, 16), ndom=(1, 2, 1))
+    with Hydro(HydroConfig(halo="fused", **kw)) as h:
+        kf = h.kernels_per_cycle()
+    with Hydro(HydroConfig(halo="kernel", **kw)) as h:
+        kk = h.kernels_per_cycle()
+    assert kk == kf + 1  # fused: no separate intra-GPU copy kernel

@@ -73,7 +73,7 @@ def run_two_ranks(kw, ncycles, timeout=240):
 
 
 def _ocfg(kw):
-    keys = ("n", "origin", "extent", "init", "user", "ndom", "cuts")
+    keys = ("n", "origin", "extent", "init", "user", "ndom", "cuts")  # halo: GPU-only option
     return OracleConfig(**{k: v for k, v in kw.items() if k in keys})
 
 
@@ -87,14 +87,17 @@ def test_two_ranks_sedov_slabs_match_oracle():
         assert rel_err(f[k], fo[k]) <= 1e-10, k
 
 
-def test_two_ranks_uneven_mixed_domains_match_oracle():
+@pytest.mark.parametrize("halo", ["fused", "kernel"])
+def test_two_ranks_uneven_mixed_domains_match_oracle(halo):
     """12 uneven domains spread over two ranks so that every domain has both same-rank
-    (intra-GPU copy) and other-rank (peer store) neighbours, incl. edge and corner slabs."""
+    (intra-GPU) and other-rank (peer store) neighbours, incl. edge and corner slabs; the ghost
+    slabs go out from the node/energy stage's epilogue (fused) or from the separate copy and
+    peer-push kernels."""
     n = (24, 20, 18)
     cuts = [[0, 5, 13, 24], [0, 7, 20], [0, 9, 18]]
     d2r = [(d * 5 + d // 3) % 2 for d in range(12)]
     kw = dict(n=n, ndom=(3, 2, 2), cuts=cuts, dom_to_rank=d2r, init="user",
-              user=jittered_state(n, 11))
+              user=jittered_state(n, 11), halo=halo)
     i0, i1, f = run_two_ranks(kw, 25)
     fo, io = oracle.run(_ocfg(kw), 25)
     assert i0["status"] == 0 and i0["dt"] == i1["dt"]
