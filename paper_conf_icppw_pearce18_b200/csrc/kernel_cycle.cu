@@ -125,7 +125,9 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   // CTA b takes [b W / G, (b+1) W / G), marched as one or two column segments.  sched_kz > 0:
   // the chunked schedule (CTA b = column b / chunks, chunk b % chunks), for A/B measurement.
   int64_t r0, r1;
+  int unit = bid, nunits = 0;  // chunked schedule: this CTA's (column, chunk) unit
   if (sched_kz > 0) {
+    nunits = ncols * ((n2 + sched_kz - 1) / sched_kz);
     const int64_t col = bid % ncols, ch = bid / ncols;  // adjacent CTAs: same z
     r0 = col * n2 + ch * sched_kz;
     r1 = col * n2 + min((int)(ch + 1) * sched_kz, n2);
@@ -269,7 +271,18 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
   uint32_t ubase = 0;  // TMA planes consumed in earlier segments (ring slot / phase continuity)
   uint32_t pbase = 0;  // plane iterations run in earlier segments (phase-barrier parity)
 
-  for (int64_t r = r0; r < r1;) {
+  for (int64_t r = r0;;) {
+  if (r >= r1) {
+    // chunked schedule on a persistent grid (fewer CTAs than units): the next unit is
+    // unit + gridDim.x, so the CTAs running at any time still hold consecutive units (adjacent
+    // columns at the same z-chunk: shared ring rows stay L2 hits)
+    if (sched_kz <= 0 || GROUP) break;
+    unit += gridDim.x;
+    if (unit >= nunits) break;
+    const int64_t c = unit % ncols, ch = unit / ncols;
+    r = c * n2 + ch * sched_kz;
+    r1 = c * n2 + min((int)(ch + 1) * sched_kz, n2);
+  }
   const int col = (int)(r / n2);
   const int k0 = (int)(r - (int64_t)col * n2);
   const int k1 = (int)min((int64_t)n2, r1 - (int64_t)col * n2);
@@ -674,16 +687,26 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
     finalize_if_last_block(st, ph, reinterpret_cast<unsigned int *>(sm + T::OFF_RED));
 }
 
-constexpr int CTX = 32, CTY = 12;
+// Node-stage tile: 32 x CTY zones (+ ring).  Two heights are compiled, 12 (512 threads) and 11
+// (480 threads); node_tile_ty picks one per domain from the wave-quantisation model below
+// (measured: 128^3 85.3 vs 89.7 us with TY = 11, weak 384^3 slabs 499.7 vs 473.8 with TY = 12).
+// The grouped launch and the one-kernel variant use CTY.
+constexpr int CTX = 32, CTY = 12, CTY_ALT = 11;
 
 // z-chunk length of the chunked schedule: minimise (waves of CTAs) x (planes per CTA incl. the
-// 2 warm-up planes).
+// 2 warm-up planes + a fixed per-chunk overhead of 1.4 plane-equivalents: pipeline fill and
+// drain, prologue).  The overhead term was fitted on the B200 at 128^3 (44 tile columns:
+// kz = 43 / 22 / 13 / 8 -> 89.5 / 97.3 / 95.0 / 109.8 us, i.e. 1 / 2 / 3 / 5 waves); without it
+// the model ties kz = 13 (3 waves x 15 planes) with kz = 43 (1 wave x 45) and took the slower.
+int64_t chunk_cost(int64_t ctas, int kz, int sms) {
+  return ((ctas + sms - 1) / sms) * (10 * (int64_t)(kz + 2) + 14);
+}
+
 int choose_kz(int tiles, int n2, int sms) {
-  int best = n2, best_cost = 1 << 30;
+  int best = n2;
+  int64_t best_cost = INT64_MAX;
   for (int kz = 4; kz <= n2; ++kz) {
-    const int chunks = (n2 + kz - 1) / kz;
-    const int waves = (tiles * chunks + sms - 1) / sms;
-    const int cost = waves * (kz + 2);
+    const int64_t cost = chunk_cost((int64_t)tiles * ((n2 + kz - 1) / kz), kz, sms);
     if (cost < best_cost) {
       best_cost = cost;
       best = kz;
@@ -692,14 +715,14 @@ int choose_kz(int tiles, int n2, int sms) {
   return std::min(best, n2);
 }
 
-template <bool FUSED>
+template <bool FUSED, int TY>
 void set_smem() {
   static bool done = false;
   if (!done) {
-    using T = CTile<CTX, CTY>;
-    cudaFuncSetAttribute(k_cycle<CTX, CTY, FUSED, false>,
+    using T = CTile<CTX, TY>;
+    cudaFuncSetAttribute(k_cycle<CTX, TY, FUSED, false>,
                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)T::BYTES);
-    if constexpr (!FUSED)
+    if constexpr (!FUSED && TY == CTY)
       cudaFuncSetAttribute(k_cycle<CTX, CTY, false, true>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)T::BYTES);
     done = true;
@@ -716,28 +739,41 @@ int num_sms() {
   return sms;
 }
 
-template <bool FUSED>
+// Modelled node-stage cost of one domain with tile height TY: best chunking's
+// chunk_cost x threads per CTA (per-plane time ~ CTA size at one CTA per SM).
+template <int TY>
+int64_t tile_cost(int n0, int n1, int n2, int sms) {
+  const int tiles = ((n0 + CTX - 1) / CTX) * ((n1 + TY - 1) / TY);
+  const int kz = choose_kz(tiles, n2, sms);
+  return chunk_cost((int64_t)tiles * ((n2 + kz - 1) / kz), kz, sms) * CTile<CTX, TY>::NTHR;
+}
+
+template <bool FUSED, int TY>
 void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st, int fold,
             const PushSlab *push, int npush, cudaStream_t s) {
-  using T = CTile<CTX, CTY>;
-  set_smem<FUSED>();
+  using T = CTile<CTX, TY>;
+  set_smem<FUSED, TY>();
   const int sms = num_sms();
-  const int tx = (d.n[0] + CTX - 1) / CTX, ty = (d.n[1] + CTY - 1) / CTY;
+  const int tx = (d.n[0] + CTX - 1) / CTX, ty = (d.n[1] + TY - 1) / TY;
   // Default: the chunked schedule (CTAs adjacent in x, y at the same z-chunk, so the tile rings
   // that neighbouring CTAs both read are L2 hits; measured faster here than the persistent
   // linearised split, which spreads concurrent CTAs over z: 94 vs 110 us at 128^3).
   // HYDRO_KZ_NODE / HYDRO_KZ_FUSED = k: chunks of k planes; = -1: the persistent split.
   static const int kz_env = getenv(FUSED ? "HYDRO_KZ_FUSED" : "HYDRO_KZ_NODE")
                                 ? atoi(getenv(FUSED ? "HYDRO_KZ_FUSED" : "HYDRO_KZ_NODE")) : 0;
+  // HYDRO_NODE_PERSIST=0: one CTA per (column, chunk) unit instead of an SM-count grid that
+  // walks the units (A/B)
+  static const int persist = getenv("HYDRO_NODE_PERSIST") ? atoi(getenv("HYDRO_NODE_PERSIST")) : 1;
   const int ncols = tx * ty;
   int G, kz = 0;
   if (kz_env >= 0) {
     kz = kz_env > 0 ? std::min(kz_env, d.n[2]) : choose_kz(ncols, d.n[2], sms);
     G = ncols * ((d.n[2] + kz - 1) / kz);
+    if (persist && !FUSED) G = std::min(G, sms);
   } else {
     G = (int)std::min<int64_t>(sms, (int64_t)ncols * d.n[2]);
   }
-  launch_pdl(k_cycle<CTX, CTY, FUSED, false>, dim3(G), dim3(T::NTHR), T::BYTES, s, maps, d, ph,
+  launch_pdl(k_cycle<CTX, TY, FUSED, false>, dim3(G), dim3(T::NTHR), T::BYTES, s, maps, d, ph,
              st, tx, ncols, kz, fold, (const NodeTask *)nullptr, 0, (const DomView *)nullptr,
              (const NodeMaps *)nullptr, push, npush);
 }
@@ -746,18 +782,32 @@ void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st
 
 size_t fused_smem_bytes() { return CTile<CTX, CTY>::BYTES; }
 int fused_box_y() { return CTile<CTX, CTY>::BYN; }
-int node_box_y() { return CTile<CTX, CTY>::BYN; }
+int node_box_y(int ty) { return ty == CTY_ALT ? CTile<CTX, CTY_ALT>::BYN : CTile<CTX, CTY>::BYN; }
 int cycle_zone_box_x() { return CTile<CTX, CTY>::ZBX; }
-int cycle_zone_box_y() { return CTile<CTX, CTY>::ZBY; }
+int cycle_zone_box_y(int ty) {
+  return ty == CTY_ALT ? CTile<CTX, CTY_ALT>::ZBY : CTile<CTX, CTY>::ZBY;
+}
+
+int node_tile_ty(int n0, int n1, int n2) {
+  // read per call (host side, at create): tests force either height within one process
+  const int force = getenv("HYDRO_NODE_TY") ? atoi(getenv("HYDRO_NODE_TY")) : 0;
+  if (force == CTY || force == CTY_ALT) return force;
+  const int sms = num_sms();
+  return tile_cost<CTY_ALT>(n0, n1, n2, sms) < tile_cost<CTY>(n0, n1, n2, sms) ? CTY_ALT : CTY;
+}
 
 void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                         int fold_finalize, cudaStream_t s) {
-  launch<true>(d, maps, ph, st, fold_finalize, nullptr, 0, s);
+  launch<true, CTY>(d, maps, ph, st, fold_finalize, nullptr, 0, s);
 }
 
 void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                        int fold_finalize, const PushSlab *push, int npush, cudaStream_t s) {
-  launch<false>(d, maps, ph, st, fold_finalize, push, npush, s);
+                        int fold_finalize, const PushSlab *push, int npush, int ty,
+                        cudaStream_t s) {
+  if (ty == CTY_ALT)
+    launch<false, CTY_ALT>(d, maps, ph, st, fold_finalize, push, npush, s);
+  else
+    launch<false, CTY>(d, maps, ph, st, fold_finalize, push, npush, s);
 }
 
 int node_group_tasks(const DomView *views_host, int n, NodeTask *out) {
@@ -766,7 +816,8 @@ int node_group_tasks(const DomView *views_host, int n, NodeTask *out) {
   const int sms = num_sms();
   int nzmax = 1;
   for (int i = 0; i < n; ++i) nzmax = std::max(nzmax, views_host[i].n[2]);
-  int best = nzmax, best_cost = INT_MAX;
+  int best = nzmax;
+  int64_t best_cost = INT64_MAX;
   for (int kz = 4; kz <= nzmax; ++kz) {
     int64_t ctas = 0;
     for (int i = 0; i < n; ++i) {
@@ -774,9 +825,9 @@ int node_group_tasks(const DomView *views_host, int n, NodeTask *out) {
       const int cols = ((d.n[0] + CTX - 1) / CTX) * ((d.n[1] + CTY - 1) / CTY);
       ctas += (int64_t)cols * ((d.n[2] + kz - 1) / kz);
     }
-    const int64_t cost = ((ctas + sms - 1) / sms) * (kz + 2);
+    const int64_t cost = chunk_cost(ctas, kz, sms);
     if (cost < best_cost) {
-      best_cost = (int)cost;
+      best_cost = cost;
       best = kz;
     }
   }
@@ -800,7 +851,7 @@ void launch_node_energy_group(const NodeTask *tasks_dev, int ntasks, int nctas,
                               const DomView *views_dev, const NodeMaps *maps_dev, const Phys &ph,
                               DevState *st, const PushSlab *push, cudaStream_t s) {
   using T = CTile<CTX, CTY>;
-  set_smem<false>();
+  set_smem<false, CTY>();
   DomView d0 = {};
   NodeMaps m0 = {};
   launch_pdl(k_cycle<CTX, CTY, false, true>, dim3(nctas), dim3(T::NTHR), T::BYTES, s, m0, d0,

@@ -125,12 +125,16 @@ void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, D
                        cudaStream_t s);
 // push/npush: this domain's fused-halo slabs (nullptr/0: none; the caller then exchanges the
 // ghost layer with launch_halo_copy / the transports).
+// ty: node-stage tile height (node_tile_ty; the TMA maps must be built with its boxes).
 void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                        int fold_finalize, const PushSlab *push, int npush, cudaStream_t s);
+                        int fold_finalize, const PushSlab *push, int npush, int ty,
+                        cudaStream_t s);
+// Node-stage tile height for a domain of n0 x n1 x n2 zones (11 or 12; HYDRO_NODE_TY forces).
+int node_tile_ty(int n0, int n1, int n2);
 int zone_box_y();
-int node_box_y();
+int node_box_y(int ty);  // node-field TMA box height of the node stage with tile height ty
 int cycle_zone_box_x();  // zone-field TMA box of the cycle kernels
-int cycle_zone_box_y();
+int cycle_zone_box_y(int ty);
 
 // End of cycle: S9 dt / time update and error latch.
 void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s);

@@ -34,6 +34,7 @@ struct LocalDom {
   DomView view[2];  // parity p reads view[p].x and writes view[p].xn
   NodeMaps maps[2];  // TMA descriptors of view[p]'s current node arrays, fused/node box
   NodeMaps zmaps[2]; // same arrays, zone-stage box
+  int node_ty = 12;  // node-stage tile height (kernel_cycle.cu node_tile_ty), sets maps' boxes
 };
 
 }  // namespace
@@ -149,8 +150,14 @@ void carve_views(void *base, const DomainBox &b, const int64_t N[3], int32_t dom
 
 namespace {
 
+bool group_node();
+
 int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
   const int64_t n0 = D.box.n[0], n1 = D.box.n[1], n2 = D.box.n[2];
+  // node-stage tile height: chosen per domain, except for the grouped node launch and the
+  // one-kernel variant, which are compiled for the default height only
+  const bool fixed_ty = h->one_kernel || (h->doms.size() > 1 && group_node());
+  D.node_ty = fixed_ty ? 12 : node_tile_ty((int)n0, (int)n1, (int)n2);
   const int64_t nsx = (n0 + 3 + 3) / 4 * 4, nsxy = nsx * (n1 + 3), nnode = nsxy * (n2 + 3);
   const int64_t zsx = (n0 + 2 + 3) / 4 * 4, zsxy = zsx * (n1 + 2);
   if (nnode >= (int64_t(1) << 31))  // the cycle kernels index a domain's storage with int32
@@ -175,7 +182,7 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
                             D.view[par].u, D.view[par].v, D.view[par].w, D.view[par].mn8};
     const double *zarr[4] = {D.view[par].m, D.view[par].e, D.view[par].P, D.view[par].mi};
     for (int kind = 0; kind < 2; ++kind) {
-      if (kind == 0 && fused_box_y() != node_box_y())
+      if (kind == 0 && D.node_ty == 12 && fused_box_y() != node_box_y(12))
         return set_err(h, HYDRO_EINVAL, "fused and node kernels must share a TMA box");
       NodeMaps &M = kind ? D.zmaps[par] : D.maps[par];
       for (int f = 0; f < 11; ++f) {
@@ -188,10 +195,10 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
         cuuint32_t box[3];
         if (zf) {
           box[0] = (cuuint32_t)cycle_zone_box_x();
-          box[1] = (cuuint32_t)cycle_zone_box_y();
+          box[1] = (cuuint32_t)cycle_zone_box_y(D.node_ty);
         } else {
           box[0] = kind ? (cuuint32_t)ZONE_BOX_X : (cuuint32_t)FUSED_BOX_X;
-          box[1] = kind ? (cuuint32_t)zone_box_y() : (cuuint32_t)fused_box_y();
+          box[1] = kind ? (cuuint32_t)zone_box_y() : (cuuint32_t)node_box_y(D.node_ty);
         }
         box[2] = 1;
         cuuint32_t es[3] = {1, 1, 1};
@@ -313,7 +320,7 @@ void launch_node_stage(hydro_ctx *h, LocalDom &D, int par, int slot, cudaStream_
   const bool p = h->fused_halo && h->push_dev[par] && h->push_count[slot] > 0;
   launch_node_energy(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h),
                      p ? h->push_dev[par] + h->push_first[slot] : nullptr,
-                     p ? h->push_count[slot] : 0, s);
+                     p ? h->push_count[slot] : 0, D.node_ty, s);
 }
 
 void launch_zone_stages(hydro_ctx *h, int par, cudaStream_t s) {

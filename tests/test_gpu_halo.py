@@ -83,3 +83,19 @@ def test_kernels_per_cycle_counts_the_fused_exchange():
     with Hydro(HydroConfig(halo="kernel", **kw)) as h:
         kk = h.kernels_per_cycle()
     assert kk == kf + 1  # fused: no separate intra-GPU copy kernel
+
+
+def test_node_tile_heights_bitwise(monkeypatch):
+    """Both compiled node-stage tile heights (kernel_cycle.cu node_tile_ty picks one per domain)
+    give the same bits: the tile shape changes which CTA computes a node, not the arithmetic."""
+    n = (45, 50, 23)
+    kw = dict(n=n, ndom=(1, 2, 1), init="user", user=jittered_state(n, 5))
+    monkeypatch.setenv("HYDRO_NODE_TY", "11")
+    fa, _ = run(12, **kw)
+    monkeypatch.setenv("HYDRO_NODE_TY", "12")
+    fb, _ = run(12, **kw)
+    for k in FIELDS:
+        assert np.array_equal(fa[k], fb[k]), k
+    fo, _ = oracle.run(_ocfg(kw), 12)
+    for k in FIELDS:
+        assert rel_err(fa[k], fo[k]) <= 1e-11, k
