@@ -286,15 +286,24 @@ __global__ void k_halo_copy(const DomView *views, const HaloCopy *chunks) {
                               (int)(p.nlo[2] - D.lo[2]));
     const int s0 = (int)S.nid((int)(p.nlo[0] - S.lo[0]), (int)(p.nlo[1] - S.lo[1]),
                               (int)(p.nlo[2] - S.lo[2]));
-    for (int t = p.start + threadIdx.x; t < p.start + p.count; t += blockDim.x) {
+    // Sources are read through the read-only path and every load of an element pair is issued
+    // before its stores (a source element is never a ghost written by this kernel, so the loads
+    // need not wait for earlier stores): two elements, twelve loads in flight per thread.
+    const int end = p.start + p.count;
+    for (int t = p.start + threadIdx.x; t < end; t += 2 * blockDim.x) {
+      const int t2 = t + blockDim.x < end ? t + blockDim.x : t;
       const int a = t % nx, r = t / nx, b = r % ny, c = r / ny;
+      const int a2 = t2 % nx, r2 = t2 / nx, b2 = r2 % ny, c2 = r2 / ny;
       const int di = d0 + c * dsxy + b * dsx + a, si = s0 + c * ssxy + b * ssx + a;
-      D.xn[di] = S.xn[si];
-      D.yn[di] = S.yn[si];
-      D.zn[di] = S.zn[si];
-      D.un[di] = S.un[si];
-      D.vn[di] = S.vn[si];
-      D.wn[di] = S.wn[si];
+      const int di2 = d0 + c2 * dsxy + b2 * dsx + a2, si2 = s0 + c2 * ssxy + b2 * ssx + a2;
+      const double v0 = __ldg(S.xn + si), v1 = __ldg(S.yn + si), v2 = __ldg(S.zn + si);
+      const double v3 = __ldg(S.un + si), v4 = __ldg(S.vn + si), v5 = __ldg(S.wn + si);
+      const double w0 = __ldg(S.xn + si2), w1 = __ldg(S.yn + si2), w2 = __ldg(S.zn + si2);
+      const double w3 = __ldg(S.un + si2), w4 = __ldg(S.vn + si2), w5 = __ldg(S.wn + si2);
+      D.xn[di] = v0; D.yn[di] = v1; D.zn[di] = v2;
+      D.un[di] = v3; D.vn[di] = v4; D.wn[di] = v5;
+      D.xn[di2] = w0; D.yn[di2] = w1; D.zn[di2] = w2;
+      D.un[di2] = w3; D.vn[di2] = w4; D.wn[di2] = w5;
     }
   } else {
     const int zx = (int)(p.zhi[0] - p.zlo[0]), zy = (int)(p.zhi[1] - p.zlo[1]);
@@ -305,7 +314,7 @@ __global__ void k_halo_copy(const DomView *views, const HaloCopy *chunks) {
                                (int)(p.zlo[2] - S.lo[2]));
     for (int t = p.start + threadIdx.x; t < p.start + p.count; t += blockDim.x) {
       const int a = t % zx, r = t / zx, b = r % zy, c = r / zy;
-      D.en[zd0 + c * zdsxy + b * zdsx + a] = S.en[zs0 + c * zssxy + b * zssx + a];
+      D.en[zd0 + c * zdsxy + b * zdsx + a] = __ldg(S.en + zs0 + c * zssxy + b * zssx + a);
     }
   }
 }

@@ -40,12 +40,11 @@ __global__ void k_peer_push(const DomView *local, const DomView *remote, const P
     const int64_t gx = p.nlo[0] + a, gy = p.nlo[1] + b, gz = p.nlo[2] + c;
     const int64_t si = S.nid((int)(gx - S.lo[0]), (int)(gy - S.lo[1]), (int)(gz - S.lo[2]));
     const int64_t di = D.nid((int)(gx - D.lo[0]), (int)(gy - D.lo[1]), (int)(gz - D.lo[2]));
-    D.xn[di] = S.xn[si];
-    D.yn[di] = S.yn[si];
-    D.zn[di] = S.zn[si];
-    D.un[di] = S.un[si];
-    D.vn[di] = S.vn[si];
-    D.wn[di] = S.wn[si];
+    // all six loads before the stores (sources are never written here: read-only path)
+    const double v0 = __ldg(S.xn + si), v1 = __ldg(S.yn + si), v2 = __ldg(S.zn + si);
+    const double v3 = __ldg(S.un + si), v4 = __ldg(S.vn + si), v5 = __ldg(S.wn + si);
+    D.xn[di] = v0; D.yn[di] = v1; D.zn[di] = v2;
+    D.un[di] = v3; D.vn[di] = v4; D.wn[di] = v5;
   }
   const int64_t zx = p.zhi[0] - p.zlo[0], zy = p.zhi[1] - p.zlo[1], zz = p.zhi[2] - p.zlo[2];
   const int64_t nzn = zx * zy * zz;
