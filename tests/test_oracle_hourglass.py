@@ -152,3 +152,21 @@ def test_sedov_with_hourglass_conserves_energy():
     assert o.step(60)["status"] == 0
     E = sum(total_energy(o.fields()))
     assert abs(E - E0) / E0 <= 1e-12
+
+
+def test_long_sedov_needs_hourglass_control():
+    """Characterisation (DESIGN.md §13 f1): without hourglass control the SG scheme lets a zone
+    next to the blast origin be crushed after ~1000 cycles (dt collapses by many orders while
+    the run is formally healthy); with kappa = 0.03 the same run keeps a normal dt.  Seen
+    identically on the GPU at 448^3 (tools/sedov_front.py).  A regression guard on the scheme's
+    behaviour, not a pin of its values."""
+    n, h = 12, 1.2 / 448
+    dts = {}
+    for kappa in (0.0, 0.03):
+        o = Oracle(OracleConfig(n=(n, n, n), extent=(h * n,) * 3, hg_coef=kappa))
+        dt0 = o.step(100)["dt"]
+        info = o.step(1200)
+        assert info["status"] == 0
+        dts[kappa] = info["dt"] / dt0
+    assert dts[0.0] < 1e-6      # collapsed
+    assert dts[0.03] > 0.1      # healthy
