@@ -99,3 +99,17 @@ def test_node_tile_heights_bitwise(monkeypatch):
     fo, _ = oracle.run(_ocfg(kw), 12)
     for k in FIELDS:
         assert rel_err(fa[k], fo[k]) <= 1e-11, k
+
+
+@pytest.mark.parametrize("k", ["1", "3"])
+def test_multi_cycle_graphs_bitwise(k, monkeypatch):
+    """hydro_step replays graphs of HYDRO_GRAPH_CYCLES cycles (default 8) plus one-cycle graphs
+    for the rest; an odd count flips the parity inside a replay.  Same bits as the default."""
+    n = (20, 18, 16)
+    kw = dict(n=n, ndom=(1, 2, 1), init="user", user=jittered_state(n, 8))
+    fd, idf = run(29, **kw)
+    monkeypatch.setenv("HYDRO_GRAPH_CYCLES", k)
+    fk, ik = run(29, **kw)
+    assert idf["cycle"] == ik["cycle"] == 29 and idf["t"] == ik["t"]
+    for f in FIELDS:
+        assert np.array_equal(fd[f], fk[f]), f
