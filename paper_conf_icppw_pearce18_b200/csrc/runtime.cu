@@ -65,6 +65,11 @@ struct hydro_ctx {
   std::vector<PushTarget> push_targets;     // local and (after peer import) remote slabs
   PushSlab *push_dev[2] = {nullptr, nullptr};
   std::vector<int32_t> push_first, push_count;  // per local slot
+  // several domains on this GPU: node/energy stages spread over nstreams streams (fork/join by
+  // events, parallel branches in the captured graph), HYDRO_NODE_STREAMS
+  int nstreams = 1;
+  cudaStream_t side[4] = {nullptr, nullptr, nullptr, nullptr};
+  cudaEvent_t fork_ev = nullptr, join_ev[4] = {nullptr, nullptr, nullptr, nullptr};
   cudaGraphExec_t graph[2] = {nullptr, nullptr};
   // graph_k cycles in one graph (per starting parity): the programmatic edges then also link one
   // cycle's finalize to the next cycle's zone stage (no graph-launch boundary between them)
@@ -344,12 +349,24 @@ bool group_node() {
 }
 
 void launch_node_stages(hydro_ctx *h, int par, cudaStream_t s) {
-  if (h->group && group_node())
+  if (h->group && group_node()) {
     launch_node_energy_group(h->ntasks_dev, (int)h->doms.size(), h->nctas, h->views_dev[par],
                              h->nmaps_dev[par], h->ph, h->st,
                              h->fused_halo ? h->push_dev[par] : nullptr, s);
-  else
+  } else if (h->nstreams > 1 && h->doms.size() > 1) {  // independent domains: parallel branches
+    cudaEventRecord(h->fork_ev, s);
+    for (int k = 1; k < h->nstreams; ++k) cudaStreamWaitEvent(h->side[k], h->fork_ev, 0);
+    for (size_t i = 0; i < h->doms.size(); ++i) {
+      const int k = (int)(i % h->nstreams);
+      launch_node_stage(h, h->doms[i], par, (int)i, k ? h->side[k] : s);
+    }
+    for (int k = 1; k < h->nstreams; ++k) {
+      cudaEventRecord(h->join_ev[k], h->side[k]);
+      cudaStreamWaitEvent(s, h->join_ev[k], 0);
+    }
+  } else {
     for (size_t i = 0; i < h->doms.size(); ++i) launch_node_stage(h, h->doms[i], par, (int)i, s);
+  }
 }
 
 // Fused-halo tables: per parity, the PushSlabs of every local source domain,
@@ -616,6 +633,18 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
   }
   if ((rc = [&]() -> int {
          CK(cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking));
+         // measured (uneven 448^3, 64 domains): 1 / 2 / 4 streams -> 12.10 / 12.71 / 12.74 G;
+         // neutral on the 4- and 8-domain configs
+         h->nstreams = 4;
+         if (const char *ns = getenv("HYDRO_NODE_STREAMS"))
+           h->nstreams = std::max(1, std::min(4, atoi(ns)));
+         if (h->nstreams > 1) {
+           CK(cudaEventCreateWithFlags(&h->fork_ev, cudaEventDisableTiming));
+           for (int k = 1; k < h->nstreams; ++k) {
+             CK(cudaStreamCreateWithFlags(&h->side[k], cudaStreamNonBlocking));
+             CK(cudaEventCreateWithFlags(&h->join_ev[k], cudaEventDisableTiming));
+           }
+         }
          CK(cudaMalloc(&h->st, sizeof(DevState)));
          DevState s0;
          std::memset(&s0, 0, sizeof(s0));
@@ -1134,6 +1163,11 @@ int hydro_destroy(hydro_ctx *h) {
   if (h->stage) cudaFree(h->stage);
   if (h->st) cudaFree(h->st);
   if (h->stream) cudaStreamDestroy(h->stream);
+  for (int k = 1; k < 4; ++k) {
+    if (h->side[k]) cudaStreamDestroy(h->side[k]);
+    if (h->join_ev[k]) cudaEventDestroy(h->join_ev[k]);
+  }
+  if (h->fork_ev) cudaEventDestroy(h->fork_ev);
   delete h;
   return HYDRO_OK;
 }
