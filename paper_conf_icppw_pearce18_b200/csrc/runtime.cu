@@ -60,6 +60,16 @@ struct hydro_ctx {
   std::vector<NodeTask> ntasks_host;
   int nctas = 0;
   int n_local_pairs = 0;
+  // halo copy overlapped with the other domains' node stages: chunks sorted by source slot, each
+  // domain's outgoing slabs copied on its own stream right after its node/energy stage
+  // (HYDRO_HALO_OVERLAP=0 for the single copy after the join, A/B)
+  // 1: per domain on its node-stage stream; 2: per domain on a dedicated halo stream; 3: per
+  // node-stage stream after its last domain (the default with <= 2 domains per stream)
+  int halo_overlap = 0;
+  cudaStream_t halo_stream = nullptr;
+  std::vector<cudaEvent_t> node_done;  // per local slot (mode 2)
+  cudaEvent_t halo_join = nullptr;
+  std::vector<int32_t> halo_first, halo_count;  // per local slot, into local_pairs_dev
   // fused halo (default two-kernel path): the node/energy stage stores the ghost slabs itself
   bool fused_halo = false;
   std::vector<PushTarget> push_targets;     // local and (after peer import) remote slabs
@@ -348,7 +358,7 @@ bool group_node() {
   return on != 0;
 }
 
-void launch_node_stages(hydro_ctx *h, int par, cudaStream_t s) {
+void launch_node_stages(hydro_ctx *h, int par, cudaStream_t s, bool with_halo = false) {
   if (h->group && group_node()) {
     launch_node_energy_group(h->ntasks_dev, (int)h->doms.size(), h->nctas, h->views_dev[par],
                              h->nmaps_dev[par], h->ph, h->st,
@@ -359,6 +369,35 @@ void launch_node_stages(hydro_ctx *h, int par, cudaStream_t s) {
     for (size_t i = 0; i < h->doms.size(); ++i) {
       const int k = (int)(i % h->nstreams);
       launch_node_stage(h, h->doms[i], par, (int)i, k ? h->side[k] : s);
+      // this domain's outgoing ghost slabs, while the other streams' node stages run: a source
+      // element is owned (never a ghost), and the destinations are next-parity ghosts that no
+      // node/energy stage writes or reads this cycle
+      if (with_halo && h->halo_overlap == 3 && i + h->nstreams >= h->doms.size()) {
+        // the last domain of this stream: copy the slabs of all of the stream's domains
+        const size_t f = (size_t)k;
+        int32_t first = -1, count = 0;
+        for (size_t j = f; j < h->doms.size(); j += h->nstreams)
+          if (h->halo_count[j] > 0) {
+            if (first < 0) first = h->halo_first[j];
+            count += h->halo_count[j];
+          }
+        if (count > 0)
+          launch_halo_copy(h->views_dev[par], h->local_pairs_dev + first, count,
+                           k ? h->side[k] : s);
+      } else if (with_halo && h->halo_overlap <= 2 && h->halo_count[i] > 0) {
+        cudaStream_t cs = k ? h->side[k] : s;
+        if (h->halo_overlap == 2) {  // the node-stage stream goes on to its next domain
+          cudaEventRecord(h->node_done[i], cs);
+          cudaStreamWaitEvent(h->halo_stream, h->node_done[i], 0);
+          cs = h->halo_stream;
+        }
+        launch_halo_copy(h->views_dev[par], h->local_pairs_dev + h->halo_first[i],
+                         h->halo_count[i], cs);
+      }
+    }
+    if (with_halo && h->halo_overlap == 2) {
+      cudaEventRecord(h->halo_join, h->halo_stream);
+      cudaStreamWaitEvent(s, h->halo_join, 0);
     }
     for (int k = 1; k < h->nstreams; ++k) {
       cudaEventRecord(h->join_ev[k], h->side[k]);
@@ -453,9 +492,10 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
       int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
     }
-    launch_node_stages(h, par, s);
+    launch_node_stages(h, par, s, h->halo_overlap);
   }
-  if (!h->fused_halo) launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
+  if (!h->fused_halo && !(h->halo_overlap && !h->split && !h->one_kernel))
+    launch_halo_copy(h->views_dev[par], h->local_pairs_dev, h->n_local_pairs, s);
   if (h->comm) {
     int rc = comm_halo(h->comm, par, s);
     if (rc) return set_err(h, rc, "halo exchange failed");
@@ -744,8 +784,40 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
              remote.push_back(P);
            }
          }
+         // chunks grouped by source slot (any order is correct: each chunk is independent)
+         // (stream of the source's node stage, source): per-domain and per-stream ranges
+         {
+           const int ns = std::max(1, h->nstreams);
+           std::stable_sort(lp.begin(), lp.end(), [ns](const HaloCopy &a, const HaloCopy &b) {
+             return a.src % ns != b.src % ns ? a.src % ns < b.src % ns : a.src < b.src;
+           });
+         }
+         h->halo_first.assign(h->doms.size(), 0);
+         h->halo_count.assign(h->doms.size(), 0);
+         for (size_t c = 0; c < lp.size(); ++c) {
+           if (h->halo_count[lp[c].src] == 0) h->halo_first[lp[c].src] = (int32_t)c;
+           ++h->halo_count[lp[c].src];
+         }
          h->n_local_pairs = (int)lp.size();  // chunk entries
          h->fused_halo = !h->split && !h->one_kernel && (cfg->flags & HYDRO_FLAG_HALO_FUSED);
+         {
+           const char *ov = getenv("HYDRO_HALO_OVERLAP");
+           // measured: per-stream copies (3) gain 0.3-0.7 % with 4 and 8 large
+           // domains; with 64 uneven domains every overlapped mode loses (a copy CTA occupies an
+           // SM's register file, so node-stage CTAs wait behind the slow sector-bound copies),
+           // and the single copy after the join stays
+           const int mode = ov ? atoi(ov) : (h->doms.size() <= 2 * (size_t)h->nstreams ? 3 : 0);
+           if (!h->fused_halo && !h->split && !h->one_kernel && !group_node() &&
+               h->nstreams > 1 && h->doms.size() > 1 && !lp.empty() && mode > 0)
+             h->halo_overlap = std::min(mode, 3);
+           if (h->halo_overlap == 2) {
+             CK(cudaStreamCreateWithFlags(&h->halo_stream, cudaStreamNonBlocking));
+             CK(cudaEventCreateWithFlags(&h->halo_join, cudaEventDisableTiming));
+             h->node_done.assign(h->doms.size(), nullptr);
+             for (cudaEvent_t &e : h->node_done)
+               CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+           }
+         }
          if (h->fused_halo) {
            int r = build_push_tables(h);
            if (r) return r;
@@ -1066,7 +1138,17 @@ int hydro_kernels_per_cycle(const hydro_ctx *h) {
   const int nd = (int)h->doms.size();
   int k = h->group ? 1 + (group_node() ? 1 : nd)
                    : (h->split ? 3 : (h->one_kernel ? 1 : 2)) * nd;  // cycle kernels
-  if (h->n_local_pairs > 0 && !h->fused_halo) k += 1;  // intra-GPU halo copy
+  if (h->halo_overlap == 3) {  // one copy per node-stage stream
+    for (int s = 0; s < h->nstreams; ++s) {
+      bool any = false;
+      for (size_t j = s; j < h->halo_count.size(); j += h->nstreams) any |= h->halo_count[j] > 0;
+      k += any;
+    }
+  } else if (h->halo_overlap) {  // one copy per source domain
+    for (int32_t c : h->halo_count) k += c > 0;
+  } else if (h->n_local_pairs > 0 && !h->fused_halo) {
+    k += 1;  // intra-GPU halo copy
+  }
   if (!fold_finalize(h)) k += 1;     // finalize
   if (h->comm) k += comm_kernels_per_cycle(h->comm);
   if (h->peer) k += peer_kernels_per_cycle(h->peer, !h->fused_halo);
@@ -1162,6 +1244,10 @@ int hydro_destroy(hydro_ctx *h) {
     if (h->push_dev[p]) cudaFree(h->push_dev[p]);
   if (h->stage) cudaFree(h->stage);
   if (h->st) cudaFree(h->st);
+  for (cudaEvent_t e : h->node_done)
+    if (e) cudaEventDestroy(e);
+  if (h->halo_join) cudaEventDestroy(h->halo_join);
+  if (h->halo_stream) cudaStreamDestroy(h->halo_stream);
   if (h->stream) cudaStreamDestroy(h->stream);
   for (int k = 1; k < 4; ++k) {
     if (h->side[k]) cudaStreamDestroy(h->side[k]);

@@ -76,13 +76,39 @@ def test_fused_halo_no_op_cycles_after_t_stop():
         assert rel_err(fg[k], fo[k]) <= 1e-10, k
 
 
-def test_kernels_per_cycle_counts_the_fused_exchange():
+def test_kernels_per_cycle_counts_the_fused_exchange(monkeypatch):
     kw = dict(n=(16, 16, 16), ndom=(1, 2, 1))
     with Hydro(HydroConfig(halo="fused", **kw)) as h:
         kf = h.kernels_per_cycle()
+    monkeypatch.setenv("HYDRO_HALO_OVERLAP", "0")
     with Hydro(HydroConfig(halo="kernel", **kw)) as h:
         kk = h.kernels_per_cycle()
     assert kk == kf + 1  # fused: no separate intra-GPU copy kernel
+    monkeypatch.setenv("HYDRO_HALO_OVERLAP", "2")
+    with Hydro(HydroConfig(halo="kernel", **kw)) as h:
+        ko = h.kernels_per_cycle()
+    assert ko == kf + 2  # overlapped: one copy per source domain
+
+
+@pytest.mark.parametrize("mode", ["1", "2", "3"])
+def test_overlapped_halo_copy_bitwise(mode, monkeypatch):
+    """Per-source-domain halo copies launched right after each domain's node/energy stage
+    (HYDRO_HALO_OVERLAP=1: on its node-stage stream; 2: on a dedicated halo stream, the
+    default) equal the single copy after the join and the undecomposed run bitwise, with more
+    domains than node-stage streams (uneven cuts, 1-zone-thick domains)."""
+    n = (24, 20, 18)
+    cuts = [[0, 5, 13, 24], [0, 1, 20], [0, 9, 10, 18]]
+    kw = dict(n=n, ndom=(3, 2, 3), cuts=cuts, init="user", user=jittered_state(n, 9),
+              halo="kernel")
+    monkeypatch.setenv("HYDRO_HALO_OVERLAP", mode)
+    fo, io = run(30, **kw)
+    monkeypatch.setenv("HYDRO_HALO_OVERLAP", "0")
+    fj, ij = run(30, **kw)
+    fs, _ = run(30, n=n, init="user", user=kw["user"])
+    assert io["status"] == 0 and io["dt"] == ij["dt"]
+    for k in FIELDS:
+        assert np.array_equal(fo[k], fj[k]), k
+        assert np.array_equal(fo[k], fs[k]), k
 
 
 def test_node_tile_heights_bitwise(monkeypatch):
