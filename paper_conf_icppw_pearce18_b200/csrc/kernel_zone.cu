@@ -32,12 +32,26 @@ constexpr int ZBX = 32, ZBY = HYDRO_ZONE_BY;           // zones per block (x, y)
 constexpr int ZNX = ZONE_BOX_X, ZNY = ZBY + 1;         // TMA node box (x padded to 16 B)
 constexpr int ZNN = ZNX * ZNY;
 constexpr int ZRS = (ZNN + 15) / 16 * 16;              // stride of one node array (128 B)
+// HYDRO_ZONE_XPBAR (default 1): the x_p ring is ordered by per-slot mbarriers (every thread
+// arrives after forming its share of plane q, a thread waits for plane p+1 only before it
+// computes zone plane p) instead of one __syncthreads per plane, so a thread may run up to one
+// plane ahead of the slowest; that needs 4 x_p slots and a 5-slot TMA ring (a slot is refilled
+// only once every thread has finished the zone plane that last read it).
+#ifndef HYDRO_ZONE_XPBAR
+#define HYDRO_ZONE_XPBAR 1
+#endif
+#if HYDRO_ZONE_XPBAR
+constexpr int ZRING = 5;                               // TMA ring: planes issued 3 ahead
+constexpr int ZXP = 4;                                 // x_p ring
+#else
 constexpr int ZRING = 4;                               // TMA ring: planes issued 3 ahead
+constexpr int ZXP = 3;
+#endif
 constexpr int ZOFF_RAW = 0;                            // [ZRING slots][6 fields][ZRS]
-constexpr int ZOFF_XP = ZOFF_RAW + ZRING * 6 * ZRS;    // [3 slots][3][ZRS]
-constexpr int ZOFF_RED = ZOFF_XP + 9 * ZRS;            // [32]
-constexpr int ZOFF_BAR = ZOFF_RED + 32;                // ZRING mbarriers
-constexpr int ZTOTAL = ZOFF_BAR + 4;
+constexpr int ZOFF_XP = ZOFF_RAW + ZRING * 6 * ZRS;    // [ZXP slots][3][ZRS]
+constexpr int ZOFF_RED = ZOFF_XP + ZXP * 3 * ZRS;      // [32]
+constexpr int ZOFF_BAR = ZOFF_RED + 32;                // ZRING + ZXP mbarriers
+constexpr int ZTOTAL = ZOFF_BAR + ZRING + ZXP;
 constexpr size_t ZBYTES = ZTOTAL * sizeof(double);
 static_assert(ZNX >= ZBX + 2, "zone-kernel TMA box too narrow (33 nodes + 1 alignment shift)");
 
@@ -59,6 +73,7 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   extern __shared__ __align__(1024) double sm[];
   double *RAW = sm + ZOFF_RAW, *XP = sm + ZOFF_XP;
   uint64_t *bar = reinterpret_cast<uint64_t *>(sm + ZOFF_BAR);
+  uint64_t *xbar = bar + ZRING;  // x_p ring (HYDRO_ZONE_XPBAR)
   pdl_wait_and_trigger();
   if ((st->halted | st->done) != 0u) return;
 
@@ -84,6 +99,7 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   if (t == 0) {
     if (smem_u32(sm) & 127u) __trap();
     for (int s = 0; s < ZRING; ++s) mbar_init(&bar[s], 1);
+    for (int s = 0; s < ZXP; ++s) mbar_init(&xbar[s], ZBX * ZBY);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
@@ -129,20 +145,43 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
       const uint32_t u = ubase + (uint32_t)(q - zk0);
       mbar_wait(&bar[u % ZRING], (u / ZRING) & 1u);
     };
+    auto xp_slot = [&](int q) {
+#if HYDRO_ZONE_XPBAR
+      return XP + ((ubase + (uint32_t)(q - zk0)) % ZXP) * 3 * ZRS;
+#else
+      return XP + ((q - zk0) % 3) * 3 * ZRS;
+#endif
+    };
     auto form_xp = [&](int q) {
       const double *R = RAW + ((ubase + (uint32_t)(q - zk0)) % ZRING) * 6 * ZRS;
-      double *X = XP + ((q - zk0) % 3) * 3 * ZRS;
+      double *X = xp_slot(q);
       for (int n = t; n < ZNN; n += ZBX * ZBY) {
         X[n] = fma(hh, R[3 * ZRS + n], R[n]);
         X[ZRS + n] = fma(hh, R[4 * ZRS + n], R[ZRS + n]);
         X[2 * ZRS + n] = fma(hh, R[5 * ZRS + n], R[2 * ZRS + n]);
       }
+#if HYDRO_ZONE_XPBAR
+      mbar_arrive(&xbar[(ubase + (uint32_t)(q - zk0)) % ZXP]);
+#endif
     };
-
+#if HYDRO_ZONE_XPBAR
+    auto xp_wait = [&](int q) {
+      const uint32_t u = ubase + (uint32_t)(q - zk0);
+      mbar_wait(&xbar[u % ZXP], (u / ZXP) & 1u);
+    };
+    if (t == 0)
+      for (int q = zk0; q < zk0 + 3 && q <= zk1; ++q) issue(q);
+    wait_plane(zk0);
+    form_xp(zk0);
+    wait_plane(zk0 + 1);  // a segment has >= 1 zone plane: node planes zk0 .. zk1 >= zk0 + 1
+    form_xp(zk0 + 1);
+    xp_wait(zk0);
+#else
     if (t == 0)
       for (int q = zk0; q < zk0 + ZRING - 1 && q <= zk1; ++q) issue(q);
     wait_plane(zk0);
     form_xp(zk0);
+#endif
 
     const bool in_xy = li < zhi.x && lj < zhi.y;
     const int64_t gx = d.lo[0] + li, gy = d.lo[1] + lj;
@@ -173,11 +212,22 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
         nx.e = ok ? d.e[(q + 1) * zsxy + zrow] : 0.0;
         nx.mi = ok ? d.mi[(q + 1) * zsxy + zrow] : 0.0;
       }
+#if HYDRO_ZONE_XPBAR
+      // every thread has formed x_p of plane p+1, so every thread has finished zone plane
+      // p-2: the TMA slot of node plane p-2 and the x_p slot of plane p-2 are free
+      xp_wait(p + 1);
+      if (t == 0 && p + 3 <= zk1) issue(p + 3);
+      if (p + 2 <= zk1) {
+        wait_plane(p + 2);
+        form_xp(p + 2);
+      }
+#else
       wait_plane(p + 1);
       form_xp(p + 1);
       __syncthreads();
       if (t == 0 && p + ZRING - 1 <= zk1) issue(p + ZRING - 1);  // slot of plane p-1 (done)
-      const double *Xa = XP + ((p - zk0) % 3) * 3 * ZRS, *Xb = XP + ((p + 1 - zk0) % 3) * 3 * ZRS;
+#endif
+      const double *Xa = xp_slot(p), *Xb = xp_slot(p + 1);
       const double *Ua = RAW + ((ubase + (uint32_t)(p - zk0)) % ZRING) * 6 * ZRS + 3 * ZRS;
       const double *Ub = RAW + ((ubase + (uint32_t)(p + 1 - zk0)) % ZRING) * 6 * ZRS + 3 * ZRS;
       double X[8], Y[8], Z[8];
