@@ -92,6 +92,7 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
   }
   const double dt = st->dt;
   const double hh = 0.5 * dt;
+  const double hgm1 = hh * ph.gm1;
   const double cfl4 = 4.0 * ph.cfl * ph.cfl, cv2 = ph.c_vol * ph.c_vol;
   double dt2min = INFINITY;
   uint32_t ubase = 0;  // planes this CTA consumed in earlier segments (mbarrier phase continuity)
@@ -194,23 +195,21 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
     // Values handed from plane p to plane p+1: the zone's m, e, 1/m (prefetched one plane
     // ahead) and its z-high face (= the z-low face of the zone above).  Two sets alternate (the
     // body runs twice per trip with the roles swapped), so no registers are copied between planes.
-    struct Carry { double m, e, mi, zx, zy, zz, za2; };
+    struct Carry { double m, e, zx, zy, zz, za2; };
     Carry S0 = {}, S1 = {};
     if (exists_xy && zk0 >= gz_lo && zk0 < gz_hi) {
       S0.m = d.m[(zk0 + 1) * zsxy + zrow];
       S0.e = d.e[(zk0 + 1) * zsxy + zrow];
-      S0.mi = d.mi[(zk0 + 1) * zsxy + zrow];
     }
 
     auto body = [&](const int p, const Carry &cu, Carry &nx) {
-      const double m = cu.m, e = cu.e, im = cu.mi;
+      const double m = cu.m, e = cu.e;
       const bool exists = exists_xy && p >= gz_lo && p < gz_hi;
       {
         const int q = p + 1;
         const bool ok = q < zk1 && exists_xy && q >= gz_lo && q < gz_hi;
         nx.m = ok ? d.m[(q + 1) * zsxy + zrow] : 0.0;
         nx.e = ok ? d.e[(q + 1) * zsxy + zrow] : 0.0;
-        nx.mi = ok ? d.mi[(q + 1) * zsxy + zrow] : 0.0;
       }
 #if HYDRO_ZONE_XPBAR
       // every thread has formed x_p of plane p+1, so every thread has finished zone plane
@@ -294,7 +293,9 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
       const double iV = frcp(V);
       const double rho = m * iV;
       const double epos = e > 0.0 ? e : 0.0;
-      const double ep = e - (hh * (ph.gm1 * rho) * epos) * DV * im;
+      // e_p = e - (hh p~ DV) / m with p~ = gm1 (m / V) e+: the mass cancels, so the zone's 1/m
+      // is not needed here (within rounding of the oracle's order)
+      const double ep = e - (hgm1 * epos) * DV * iV;
       const double eppos = ep > 0.0 ? ep : 0.0;
       const double pr = ph.gm1 * rho * eppos;
       const double c2 = ph.ggm1 * eppos;
