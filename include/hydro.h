@@ -160,6 +160,22 @@ int hydro_get_box(hydro_ctx *h, const int64_t lo[3], const int64_t hi[3], uint32
 int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, double t,
                     double dt);
 
+/* Streamed batches of independent runs on this context's mesh (an ensemble: many initial
+   states through the same cycle).  Batch b starts from the host state in[7b .. 7b+6] = x, y, z,
+   u, v, w (global node arrays) and e (global zone array), laid out as for hydro_set_state,
+   with clock t0[b], dt0[b] and cycle 0; it runs ncycles cycles (the hot path of hydro_step)
+   and writes x, y, z, u, v, w, e after them into out[7b .. 7b+6] (as hydro_get_fields).  Zone
+   masses are the context's, as for hydro_set_state.  The host->device copy of batch b+1 and
+   the device->host copy of batch b-1 run on two copy streams while batch b computes (two
+   device staging slots each way, allocated on first use and kept until hydro_destroy), so for
+   page-locked host buffers the transfers hide behind the cycles.  info (NULL or nbatch
+   entries) receives each batch's final clock and status; the return value is the first
+   nonzero batch status (a physics error ends only that batch's cycles, later batches still
+   run), HYDRO_EINVAL for bad arguments or a multi-rank context (nranks > 1), HYDRO_ECUDA.
+   Synchronous on return; the context then holds the last batch's state.  Not collective. */
+int hydro_run_batch(hydro_ctx *h, int32_t nbatch, int32_t ncycles, const double *const *in,
+                    double *const *out, const double *t0, const double *dt0, hydro_info *info);
+
 /* Peer transport (HYDRO_FLAG_PEER) bootstrap, collective: after hydro_create every rank calls
    hydro_peer_export (buf NULL: *len = bytes needed), the caller all-gathers the records (padded to
    a common len_per_rank, rank order), and every rank calls hydro_peer_import with all of them;

@@ -143,6 +143,9 @@ void launch_finalize(DevState *st, const Phys &ph, cudaStream_t s);
 void launch_halo_copy(const DomView *views_dev, const HaloCopy *chunks_dev, int nchunks,
                       cudaStream_t s);
 
+// hydro_run_batch: t, dt, cycle 0, errors cleared (one thread).
+void launch_reset_clock(DevState *st, double t, double dt, unsigned done, cudaStream_t s);
+
 // Strided 3-D box copy (src/dst pre-offset to the box origin; pitches in elements).
 void launch_copy3d(const double *src, int64_t ssx, int64_t ssxy, double *dst, int64_t dsx,
                    int64_t dsxy, int ex, int ey, int ez, cudaStream_t s);

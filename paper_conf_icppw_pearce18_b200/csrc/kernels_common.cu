@@ -377,6 +377,20 @@ void launch_finalize_init(DevState *st, double dt_first, double dt_init, double 
                           double t_stop, double t0, cudaStream_t s) {
   k_finalize_init<<<1, 1, 0, s>>>(st, dt_first, dt_init, dt_max, t_stop, t0);
 }
+// hydro_run_batch: a fresh clock for the next batch (t, dt given; cycle 0; errors cleared).
+__global__ void k_reset_clock(DevState *st, double t, double dt, unsigned done) {
+  st->t = t;
+  st->dt = dt;
+  st->cycle = 0;
+  st->err = 0;
+  st->halted = 0;
+  st->done = done;
+  st->bad_zone = ~0ull;
+  st->dtz_acc = (unsigned long long)__double_as_longlong(INFINITY);
+}
+void launch_reset_clock(DevState *st, double t, double dt, unsigned done, cudaStream_t s) {
+  k_reset_clock<<<1, 1, 0, s>>>(st, t, dt, done);
+}
 void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
   k_zone_split<<<grid_for(d.n[0] + 2, d.n[1] + 2, d.n[2] + 2), dim3(BX, BY), 0, s>>>(d, ph, st);
 }

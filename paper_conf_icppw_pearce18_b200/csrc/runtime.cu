@@ -92,6 +92,13 @@ struct hydro_ctx {
   int failed = 0;
   Comm *comm = nullptr;
   Peer *peer = nullptr;      // HYDRO_FLAG_PEER transport (nranks > 1)
+  // hydro_run_batch: two device staging slots each for the dense global inputs and outputs
+  // (x,y,z,u,v,w on nodes, e on zones), two copy streams and their slot events (lazy)
+  double *bin[2] = {nullptr, nullptr}, *bout[2] = {nullptr, nullptr};
+  cudaStream_t cp_in = nullptr, cp_out = nullptr;
+  cudaEvent_t in_ready[2] = {}, in_free[2] = {}, out_ready[2] = {}, out_free[2] = {};
+  DevState *bst = nullptr;  // per-batch final DevState
+  int32_t bst_cap = 0;
   double *stage = nullptr;  // contiguous device staging for host transfers (lazy)
   size_t stage_cap = 0;
   std::string err;
@@ -1133,6 +1140,179 @@ int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, 
   return HYDRO_OK;
 }
 
+namespace {
+// Dense global staging <-> the local domains of parity par, on stream s (hydro_run_batch).
+// Scatter: owned + ghost entries, as upload_state; gather: the lowest-index owner of each node
+// and every owned zone, as hydro_get_box.  Field f of the dense block: nodes f*NnG, e at 6*NnG.
+void batch_scatter(hydro_ctx *h, const double *dense, int par, cudaStream_t s) {
+  const int64_t gn[3] = {h->L.N[0] + 1, h->L.N[1] + 1, h->L.N[2] + 1};
+  const int64_t gz[3] = {h->L.N[0], h->L.N[1], h->L.N[2]};
+  const int64_t NnG = gn[0] * gn[1] * gn[2];
+  for (LocalDom &D : h->doms) {
+    const DomView &v = D.view[par];
+    int64_t nlo[3], next[3], nloc[3], zlo[3], zext[3], zloc[3];
+    for (int a = 0; a < 3; ++a) {
+      const int64_t lo = std::max<int64_t>(D.box.lo[a] - 1, 0);
+      const int64_t hi = std::min<int64_t>(D.box.lo[a] + D.box.n[a] + 1, h->L.N[a]);
+      nlo[a] = lo; next[a] = hi - lo + 1; nloc[a] = lo - D.box.lo[a] + 1;
+      zlo[a] = lo; zext[a] = hi - lo; zloc[a] = nloc[a];
+    }
+    double *dst[7] = {const_cast<double *>(v.x), const_cast<double *>(v.y),
+                      const_cast<double *>(v.z), const_cast<double *>(v.u),
+                      const_cast<double *>(v.v), const_cast<double *>(v.w),
+                      const_cast<double *>(v.e)};
+    for (int f = 0; f < 7; ++f) {
+      const bool z = f == 6;
+      const int64_t *g = z ? gz : gn, *lo = z ? zlo : nlo, *ex = z ? zext : next,
+                    *lc = z ? zloc : nloc;
+      const int64_t dsx = z ? v.zsx : v.nsx, dsxy = z ? v.zsxy : v.nsxy;
+      const double *src = dense + f * NnG + (lo[2] * g[1] + lo[1]) * g[0] + lo[0];
+      launch_copy3d(src, g[0], g[0] * g[1], dst[f] + (lc[2] * (dsxy / dsx) + lc[1]) * dsx + lc[0],
+                    dsx, dsxy, (int)ex[0], (int)ex[1], (int)ex[2], s);
+    }
+  }
+}
+void batch_gather(hydro_ctx *h, double *dense, int par, cudaStream_t s) {
+  const int64_t gn[3] = {h->L.N[0] + 1, h->L.N[1] + 1, h->L.N[2] + 1};
+  const int64_t gz[3] = {h->L.N[0], h->L.N[1], h->L.N[2]};
+  const int64_t NnG = gn[0] * gn[1] * gn[2];
+  for (LocalDom &D : h->doms) {
+    const DomView &v = D.view[par];
+    int64_t nlo[3], next[3], zlo[3], zext[3];
+    for (int a = 0; a < 3; ++a) {
+      nlo[a] = D.box.lo[a] + (D.box.idx[a] > 0 ? 1 : 0);
+      next[a] = D.box.lo[a] + D.box.n[a] - nlo[a] + 1;
+      zlo[a] = D.box.lo[a];
+      zext[a] = D.box.n[a];
+    }
+    const double *src[7] = {v.x, v.y, v.z, v.u, v.v, v.w, v.e};
+    for (int f = 0; f < 7; ++f) {
+      const bool z = f == 6;
+      const int64_t *g = z ? gz : gn, *lo = z ? zlo : nlo, *ex = z ? zext : next;
+      const int64_t dsx = z ? v.zsx : v.nsx, dsxy = z ? v.zsxy : v.nsxy;
+      int64_t lc[3];
+      for (int a = 0; a < 3; ++a) lc[a] = lo[a] - D.box.lo[a] + 1;
+      launch_copy3d(src[f] + (lc[2] * (dsxy / dsx) + lc[1]) * dsx + lc[0], dsx, dsxy,
+                    dense + f * NnG + (lo[2] * g[1] + lo[1]) * g[0] + lo[0], g[0], g[0] * g[1],
+                    (int)ex[0], (int)ex[1], (int)ex[2], s);
+    }
+  }
+}
+}  // namespace
+
+int hydro_run_batch(hydro_ctx *h, int32_t nbatch, int32_t ncycles, const double *const *in,
+                    double *const *out, const double *t0, const double *dt0, hydro_info *info) {
+  if (!h || nbatch < 0 || ncycles < 0 || (nbatch > 0 && (!in || !out || !t0 || !dt0)))
+    return set_err(h, HYDRO_EINVAL, "run_batch: bad argument");
+  if (h->cfg.nranks > 1 || h->peer || h->comm)
+    return set_err(h, HYDRO_EINVAL, "run_batch: single-rank contexts only");
+  for (int32_t b = 0; b < nbatch; ++b) {
+    if (!(dt0[b] > 0.0) || !std::isfinite(t0[b]))
+      return set_err(h, HYDRO_EINVAL, "run_batch: bad t0/dt0");
+    for (int f = 0; f < 7; ++f)
+      if (!in[7 * b + f] || !out[7 * b + f])
+        return set_err(h, HYDRO_EINVAL, "run_batch: missing array");
+  }
+  if (nbatch == 0) return HYDRO_OK;
+  CK(cudaSetDevice(h->device));
+  const int64_t NnG = (h->L.N[0] + 1) * (h->L.N[1] + 1) * (h->L.N[2] + 1);
+  const int64_t NzG = h->L.N[0] * h->L.N[1] * h->L.N[2];
+  const size_t nbytes = (size_t)NnG * sizeof(double), zbytes = (size_t)NzG * sizeof(double);
+  if (!h->cp_in) {
+    CK(cudaStreamCreateWithFlags(&h->cp_in, cudaStreamNonBlocking));
+    CK(cudaStreamCreateWithFlags(&h->cp_out, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i) {
+      CK(cudaMalloc(&h->bin[i], 6 * nbytes + zbytes));
+      CK(cudaMalloc(&h->bout[i], 6 * nbytes + zbytes));
+      for (cudaEvent_t *e : {&h->in_ready[i], &h->in_free[i], &h->out_ready[i], &h->out_free[i]})
+        CK(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
+    }
+  }
+  if (nbatch > h->bst_cap) {
+    if (h->bst) CK(cudaFree(h->bst));
+    CK(cudaMalloc(&h->bst, sizeof(DevState) * nbatch));
+    h->bst_cap = nbatch;
+  }
+  cudaStream_t s = h->stream;
+  // the copy streams start after everything already enqueued on the compute stream
+  CK(cudaEventRecord(h->in_free[0], s));
+  CK(cudaStreamWaitEvent(h->cp_in, h->in_free[0], 0));
+  CK(cudaStreamWaitEvent(h->cp_out, h->in_free[0], 0));
+  CK(cudaEventRecord(h->in_free[0], h->cp_in));
+  CK(cudaEventRecord(h->in_free[1], h->cp_in));
+  CK(cudaEventRecord(h->out_free[0], h->cp_out));
+  CK(cudaEventRecord(h->out_free[1], h->cp_out));
+  auto h2d = [&](int32_t b) -> int {  // batch b's inputs into staging slot b & 1 (copy-in stream)
+    const int k = b & 1;
+    CK(cudaStreamWaitEvent(h->cp_in, h->in_free[k], 0));
+    for (int f = 0; f < 7; ++f)
+      CK(cudaMemcpyAsync(h->bin[k] + f * NnG, in[7 * b + f], f < 6 ? nbytes : zbytes,
+                         cudaMemcpyHostToDevice, h->cp_in));
+    CK(cudaEventRecord(h->in_ready[k], h->cp_in));
+    return HYDRO_OK;
+  };
+  int rc = h2d(0);
+  if (rc) return rc;
+  for (int32_t b = 0; b < nbatch; ++b) {
+    const int k = b & 1;
+    // the copy-in of batch b+1 overlaps batch b's cycles
+    if (b + 1 < nbatch && (rc = h2d(b + 1))) return rc;
+    CK(cudaStreamWaitEvent(s, h->in_ready[k], 0));
+    batch_scatter(h, h->bin[k], h->parity, s);
+    CK(cudaEventRecord(h->in_free[k], s));
+    const unsigned done = (h->ph.t_stop > 0.0 && t0[b] >= h->ph.t_stop) ? 1u : 0u;
+    launch_reset_clock(h->st, t0[b], dt0[b], done, s);
+    for (int32_t c = 0; c < ncycles;) {
+      if (h->use_graph && h->graph_k > 1 && ncycles - c >= h->graph_k) {
+        CK(cudaGraphLaunch(h->graphk[h->parity], s));
+        h->parity ^= h->graph_k & 1;
+        c += h->graph_k;
+        continue;
+      }
+      if (h->use_graph) {
+        CK(cudaGraphLaunch(h->graph[h->parity], s));
+      } else if ((rc = enqueue_cycle(h, h->parity, s))) {
+        return rc;
+      }
+      h->parity ^= 1;
+      ++c;
+    }
+    CK(cudaMemcpyAsync(h->bst + b, h->st, sizeof(DevState), cudaMemcpyDeviceToDevice, s));
+    // results into staging slot k once its previous copy-out is done; the copy-out of batch b
+    // overlaps batch b+1's cycles
+    CK(cudaStreamWaitEvent(s, h->out_free[k], 0));
+    batch_gather(h, h->bout[k], h->parity, s);
+    CK(cudaEventRecord(h->out_ready[k], s));
+    CK(cudaStreamWaitEvent(h->cp_out, h->out_ready[k], 0));
+    for (int f = 0; f < 7; ++f)
+      CK(cudaMemcpyAsync(out[7 * b + f], h->bout[k] + f * NnG, f < 6 ? nbytes : zbytes,
+                         cudaMemcpyDeviceToHost, h->cp_out));
+    CK(cudaEventRecord(h->out_free[k], h->cp_out));
+  }
+  CK(cudaStreamSynchronize(h->cp_out));
+  CK(cudaStreamSynchronize(s));
+  std::vector<DevState> fin(nbatch);
+  CK(cudaMemcpy(fin.data(), h->bst, sizeof(DevState) * nbatch, cudaMemcpyDeviceToHost));
+  int status = HYDRO_OK;
+  for (int32_t b = 0; b < nbatch; ++b) {
+    int sb = HYDRO_OK;
+    if (fin[b].halted & ERR_TANGLED) sb = HYDRO_ETANGLED;
+    else if (fin[b].halted & ERR_NONFINITE) sb = HYDRO_ENONFINITE;
+    if (info) {
+      info[b].t = fin[b].t;
+      info[b].dt = fin[b].dt;
+      info[b].cycle = (int64_t)fin[b].cycle;
+      info[b].dt_min_zone = fin[b].dtz_last;
+      info[b].status = sb;
+      info[b].bad_zone = (fin[b].bad_zone == ~0ull) ? -1 : (int64_t)fin[b].bad_zone;
+    }
+    if (status == HYDRO_OK) status = sb;
+  }
+  // the context continues from the last batch's state (its clock is on the device already)
+  h->failed = 0;
+  return status;
+}
+
 int hydro_kernels_per_cycle(const hydro_ctx *h) {
   if (!h) return HYDRO_EINVAL;
   const int nd = (int)h->doms.size();
@@ -1248,6 +1428,15 @@ int hydro_destroy(hydro_ctx *h) {
     if (e) cudaEventDestroy(e);
   if (h->halo_join) cudaEventDestroy(h->halo_join);
   if (h->halo_stream) cudaStreamDestroy(h->halo_stream);
+  for (int i = 0; i < 2; ++i) {
+    if (h->bin[i]) cudaFree(h->bin[i]);
+    if (h->bout[i]) cudaFree(h->bout[i]);
+    for (cudaEvent_t e : {h->in_ready[i], h->in_free[i], h->out_ready[i], h->out_free[i]})
+      if (e) cudaEventDestroy(e);
+  }
+  if (h->bst) cudaFree(h->bst);
+  if (h->cp_in) cudaStreamDestroy(h->cp_in);
+  if (h->cp_out) cudaStreamDestroy(h->cp_out);
   if (h->stream) cudaStreamDestroy(h->stream);
   for (int k = 1; k < 4; ++k) {
     if (h->side[k]) cudaStreamDestroy(h->side[k]);

@@ -84,6 +84,10 @@ def load_library(path: str = LIB_PATH) -> C.CDLL:
     L.hydro_set_state.argtypes = [C.c_void_p, C.POINTER(C.POINTER(C.c_double)),
                                   C.POINTER(C.c_double), C.c_double, C.c_double]
     L.hydro_get_info.argtypes = [C.c_void_p, C.POINTER(HydroInfoC)]
+    L.hydro_run_batch.argtypes = [C.c_void_p, C.c_int32, C.c_int32,
+                                  C.POINTER(C.POINTER(C.c_double)),
+                                  C.POINTER(C.POINTER(C.c_double)), C.POINTER(C.c_double),
+                                  C.POINTER(C.c_double), C.POINTER(HydroInfoC)]
     L.hydro_destroy.argtypes = [C.c_void_p]
     L.hydro_layout_export.argtypes = [C.POINTER(HydroConfigC), C.POINTER(C.c_int64),
                                       C.POINTER(C.c_size_t)]
@@ -541,6 +545,36 @@ class Hydro:
                                      float(t), float(dt))
         if rc != 0:
             raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+
+    def run_batch(self, states: Sequence[Dict[str, np.ndarray]], ncycles: int,
+                  t0: Sequence[float], dt0: Sequence[float],
+                  out: Optional[Sequence[Dict[str, np.ndarray]]] = None):
+        """hydro_run_batch: independent runs from the host states ``states[b]`` (x, y, z, u, v,
+        w on nodes and e on zones, global arrays), ncycles each, with the host<->device copies
+        of neighbouring batches overlapped with the cycles (pin the arrays for the overlap).
+        Returns (outputs, infos); ``out`` may supply caller-owned (pinned) result arrays."""
+        nb = len(states)
+        nx, ny, nz = (int(v) for v in self.cfg.n)
+        names = NODE_FIELDS + ("e",)
+        ins = [[np.ascontiguousarray(st[k], dtype=np.float64) for k in names] for st in states]
+        if out is None:
+            out = [{k: np.empty((nz + 1, ny + 1, nx + 1) if k != "e" else (nz, ny, nx))
+                    for k in names} for _ in range(nb)]
+        P = C.POINTER(C.c_double)
+        for b in range(nb):
+            for k in names:
+                a = out[b][k]
+                if a.dtype != np.float64 or not a.flags.c_contiguous:
+                    raise ValueError("run_batch: out arrays must be C-contiguous float64")
+        pin = (P * (7 * nb))(*[a.ctypes.data_as(P) for row in ins for a in row])
+        pout = (P * (7 * nb))(*[out[b][k].ctypes.data_as(P) for b in range(nb) for k in names])
+        ct0 = (C.c_double * nb)(*[float(v) for v in t0])
+        cdt0 = (C.c_double * nb)(*[float(v) for v in dt0])
+        infos = (HydroInfoC * max(nb, 1))()
+        rc = self._L.hydro_run_batch(self._h, nb, int(ncycles), pin, pout, ct0, cdt0, infos)
+        if rc in (-3, -1):
+            raise HydroError(rc, self._L.hydro_last_error(self._h).decode())
+        return out, [_info(infos[b]) for b in range(nb)]
 
     def close(self):
         if getattr(self, "_h", None):
