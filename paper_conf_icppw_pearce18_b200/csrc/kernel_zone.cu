@@ -4,11 +4,12 @@
 // half-step positions x_p = x + dt/2 u (S1), face and corner vectors, V, DV (S2), the energy
 // predictor and EOS (S3), the artificial viscosity and P = p + q (S4), and dt_z (S6, owned zones
 // only, reduced per block and combined with one atomicMin).  P is written to HBM (8 B/zone) for
-// the node/energy kernel (kernel_node.cu).  A 32x8 block marches a z-chunk; node planes stream in
-// by TMA into a 3-slot ring one plane ahead of use, x_p is formed once per node into a 3-slot
-// ring, and a single __syncthreads per plane orders the rings.  No redundant compute: this is the
-// point of the split versus the one-kernel variant (kernel_fused.cu), which recomputes a zone
-// ring per tile.
+// the node/energy kernel (kernel_cycle.cu).  A 32x8 block marches its share of z-columns; node
+// planes stream in by TMA into a 5-slot ring three planes ahead of use, x_p is formed once per
+// node into a 4-slot ring ordered by per-slot mbarriers (HYDRO_ZONE_XPBAR; the older variant
+// orders a 3-slot ring with one __syncthreads per plane).  No redundant compute: this is the
+// point of the split versus the one-kernel variant (k_cycle<..., FUSED>), which recomputes a
+// zone ring per tile.
 #include <algorithm>
 #include <cmath>
 #include <cstdlib>
