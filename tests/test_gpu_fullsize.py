@@ -32,7 +32,7 @@ WINDOWS = [((56, 100, 200), (72, 116, 216)),   # x cut at 64
            ((440, 440, 440), (448, 448, 448))]  # far corner (walls)
 
 
-def _state():
+def _state(N=N):
     s = user_state((N, N, N), extent=(1.2, 1.2, 1.2))
     L = 1.2
     x, y, z = s["x"], s["y"], s["z"]
@@ -47,10 +47,10 @@ def _state():
     return s
 
 
-def _run(s, **kw):
+def _run(s, N=N, windows=WINDOWS, **kw):
     with Hydro(HydroConfig(n=(N, N, N), init="user", user=s, **kw)) as h:
         info = h.step(CYCLES)
-        boxes = [h.box(lo, hi) for lo, hi in WINDOWS]
+        boxes = [h.box(lo, hi) for lo, hi in windows]
     return info, boxes
 
 
@@ -64,3 +64,25 @@ def test_uneven448_sixty_four_domains_equal_single_domain_bitwise():
         for k in bd:
             assert np.array_equal(bd[k], bo[k]), (lo, hi, k)
         assert np.abs(bd["u"]).max() > 0.0 and np.abs(bd["q"]).max() >= 0.0
+
+
+W384 = [((100, 88, 150), (116, 104, 166)),    # y cut at 96
+        ((0, 184, 0), (16, 200, 16)),          # y cut at 192, on the -x/-z walls
+        ((368, 280, 368), (384, 296, 384)),    # y cut at 288, on the +x/+z walls
+        ((200, 376, 10), (216, 384, 26))]      # +y wall
+
+
+def test_weak384_four_y_slabs_equal_single_domain_bitwise():
+    """BASELINE config 4 at N=1 in bench.py's launch configuration (384^3 as four 384x96x384
+    y-slabs on one GPU: grouped zone stage, node stages on four streams, per-stream halo copies
+    overlapped with the other streams' node stages) equals the single-domain run bit for bit
+    around every cut, from the smooth moving state."""
+    n = 384
+    s = _state(n)
+    i_dec, b_dec = _run(s, N=n, windows=W384, ndom=(1, 4, 1))
+    i_one, b_one = _run(s, N=n, windows=W384)
+    assert i_dec["status"] == 0 and i_dec["cycle"] == CYCLES
+    assert i_dec["t"] == i_one["t"] and i_dec["dt"] == i_one["dt"]
+    for (lo, hi), bd, bo in zip(W384, b_dec, b_one):
+        for k in bd:
+            assert np.array_equal(bd[k], bo[k]), (lo, hi, k)
