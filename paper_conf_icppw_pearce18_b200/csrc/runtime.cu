@@ -78,6 +78,10 @@ struct hydro_ctx {
   // several domains on this GPU: node/energy stages spread over nstreams streams (fork/join by
   // events, parallel branches in the captured graph), HYDRO_NODE_STREAMS
   int nstreams = 1;
+  // launch order of the local domains' node stages and the stream of each (HYDRO_NODE_LPT=1,
+  // default: largest first, each onto the least-loaded stream; 0: index order, round-robin)
+  std::vector<int32_t> node_order, node_stream;
+  std::vector<size_t> stream_last;  // position in node_order of each stream's last domain
   cudaStream_t side[4] = {nullptr, nullptr, nullptr, nullptr};
   cudaEvent_t fork_ev = nullptr, join_ev[4] = {nullptr, nullptr, nullptr, nullptr};
   cudaGraphExec_t graph[2] = {nullptr, nullptr};
@@ -373,19 +377,20 @@ void launch_node_stages(hydro_ctx *h, int par, cudaStream_t s, bool with_halo = 
   } else if (h->nstreams > 1 && h->doms.size() > 1) {  // independent domains: parallel branches
     cudaEventRecord(h->fork_ev, s);
     for (int k = 1; k < h->nstreams; ++k) cudaStreamWaitEvent(h->side[k], h->fork_ev, 0);
-    for (size_t i = 0; i < h->doms.size(); ++i) {
-      const int k = (int)(i % h->nstreams);
+    for (size_t oi = 0; oi < h->node_order.size(); ++oi) {
+      const size_t i = (size_t)h->node_order[oi];
+      const int k = h->node_stream[i];
       launch_node_stage(h, h->doms[i], par, (int)i, k ? h->side[k] : s);
       // this domain's outgoing ghost slabs, while the other streams' node stages run: a source
       // element is owned (never a ghost), and the destinations are next-parity ghosts that no
       // node/energy stage writes or reads this cycle
-      if (with_halo && h->halo_overlap == 3 && i + h->nstreams >= h->doms.size()) {
-        // the last domain of this stream: copy the slabs of all of the stream's domains
-        const size_t f = (size_t)k;
+      if (with_halo && h->halo_overlap == 3 && h->stream_last[k] == oi) {
+        // the last domain of this stream: copy the slabs of all of the stream's domains (one
+        // contiguous range: the chunks are sorted by (stream, source))
         int32_t first = -1, count = 0;
-        for (size_t j = f; j < h->doms.size(); j += h->nstreams)
-          if (h->halo_count[j] > 0) {
-            if (first < 0) first = h->halo_first[j];
+        for (size_t j = 0; j < h->doms.size(); ++j)
+          if (h->node_stream[j] == k && h->halo_count[j] > 0) {
+            if (first < 0 || h->halo_first[j] < first) first = h->halo_first[j];
             count += h->halo_count[j];
           }
         if (count > 0)
@@ -792,11 +797,39 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
            }
          }
          // chunks grouped by source slot (any order is correct: each chunk is independent)
-         // (stream of the source's node stage, source): per-domain and per-stream ranges
+         // node-stage streams: LPT on the domain sizes (largest first onto the least-loaded
+         // stream), launched largest first, so small domains fill the other streams' tails
          {
+           const size_t nd = h->doms.size();
            const int ns = std::max(1, h->nstreams);
-           std::stable_sort(lp.begin(), lp.end(), [ns](const HaloCopy &a, const HaloCopy &b) {
-             return a.src % ns != b.src % ns ? a.src % ns < b.src % ns : a.src < b.src;
+           const char *lpt_env = getenv("HYDRO_NODE_LPT");
+           const bool lpt = !lpt_env || atoi(lpt_env) != 0;
+           h->node_order.resize(nd);
+           h->node_stream.assign(nd, 0);
+           for (size_t i = 0; i < nd; ++i) h->node_order[i] = (int32_t)i;
+           auto zones = [&](int32_t i) {
+             const DomainBox &b = h->doms[i].box;
+             return (int64_t)b.n[0] * b.n[1] * b.n[2];
+           };
+           if (lpt) {
+             std::stable_sort(h->node_order.begin(), h->node_order.end(),
+                              [&](int32_t a, int32_t b) { return zones(a) > zones(b); });
+             std::vector<int64_t> load(ns, 0);
+             for (int32_t i : h->node_order) {
+               const int k = (int)(std::min_element(load.begin(), load.end()) - load.begin());
+               h->node_stream[i] = k;
+               load[k] += zones(i);
+             }
+           } else {
+             for (size_t i = 0; i < nd; ++i) h->node_stream[i] = (int32_t)(i % ns);
+           }
+           h->stream_last.assign(ns, (size_t)-1);
+           for (size_t oi = 0; oi < nd; ++oi) h->stream_last[h->node_stream[h->node_order[oi]]] = oi;
+           // halo chunks sorted by (stream of the source's node stage, source): per-domain and
+           // per-stream ranges
+           std::stable_sort(lp.begin(), lp.end(), [h](const HaloCopy &a, const HaloCopy &b) {
+             const int sa = h->node_stream[a.src], sb = h->node_stream[b.src];
+             return sa != sb ? sa < sb : a.src < b.src;
            });
          }
          h->halo_first.assign(h->doms.size(), 0);
@@ -1321,7 +1354,8 @@ int hydro_kernels_per_cycle(const hydro_ctx *h) {
   if (h->halo_overlap == 3) {  // one copy per node-stage stream
     for (int s = 0; s < h->nstreams; ++s) {
       bool any = false;
-      for (size_t j = s; j < h->halo_count.size(); j += h->nstreams) any |= h->halo_count[j] > 0;
+      for (size_t j = 0; j < h->halo_count.size(); ++j)
+        any |= h->node_stream[j] == s && h->halo_count[j] > 0;
       k += any;
     }
   } else if (h->halo_overlap) {  // one copy per source domain
