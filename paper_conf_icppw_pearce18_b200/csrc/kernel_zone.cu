@@ -119,10 +119,18 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
     const int tcols = T.tcols;
     const int nplanes = zhi.z - zlo.z;
     const int64_t rl = r - T.u0, rl1 = min(r1, T.u0 + T.units) - T.u0;  // task-local units
-    const int col = (int)(rl / nplanes);
-    const int zk0 = zlo.z + (int)(rl - (int64_t)col * nplanes);
-    const int zk1 = zlo.z + (int)min((int64_t)nplanes, rl1 - (int64_t)col * nplanes);
-    r = T.u0 + (int64_t)col * nplanes + (zk1 - zlo.z);
+    // unit order: z-blocks of zblk planes, within a block column-major (zblk = nplanes: plain
+    // column-major), so CTAs that run at the same time march neighbouring columns over the same
+    // z range and the node-box rows the columns share are L2 hits
+    const int zblk = T.zblk;
+    const int64_t bsz = (int64_t)(T.units / nplanes) * zblk;  // units of a full z-block
+    const int zb = (int)(rl / bsz);
+    const int lb = min(zblk, nplanes - zb * zblk);
+    const int64_t rem = rl - (int64_t)zb * bsz;
+    const int col = (int)(rem / lb);
+    const int zk0 = zlo.z + zb * zblk + (int)(rem - (int64_t)col * lb);
+    const int zk1 = zlo.z + zb * zblk + (int)min((int64_t)lb, rl1 - (int64_t)zb * bsz - (int64_t)col * lb);
+    r = T.u0 + (int64_t)zb * bsz + (int64_t)col * lb + (zk1 - zlo.z - zb * zblk);
     const int gz_lo = -(int)d.lo[2], gz_hi = d.N[2] - (int)d.lo[2];
     // this segment's zones: local [zi0, zi0+32) x [zj0, zj0+8) x [zk0, zk1) inside [zlo, zhi):
     // the owned zones plus the ghost ring where a neighbour domain exists (ghost zones beyond
@@ -347,6 +355,9 @@ ZoneTask zone_task(const DomView &d, int slot) {
   const int ty = (T.zhi[1] - T.zlo[1] + ZBY - 1) / ZBY;
   T.units = (int64_t)T.tcols * ty * (T.zhi[2] - T.zlo[2]);
   T.u0 = 0;
+  T.zblk = T.zhi[2] - T.zlo[2];
+  static const int zb_env = getenv("HYDRO_ZONE_ZBLK") ? atoi(getenv("HYDRO_ZONE_ZBLK")) : 0;
+  if (zb_env > 0) T.zblk = std::min(T.zblk, zb_env);
   return T;
 }
 
@@ -372,7 +383,7 @@ int zone_box_y() { return ZNY; }
 void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                        cudaStream_t s) {
   const int slots = zone_slots();
-  const ZoneTask T = zone_task(d, 0);
+  ZoneTask T = zone_task(d, 0);
   // Default: the persistent linearised split (measured 67 vs 70 us for the best chunking at
   // 128^3).  HYDRO_KZ_ZONE=k: the chunked schedule with k planes per CTA (A/B measurement).
   static const int kz_env = getenv("HYDRO_KZ_ZONE") ? atoi(getenv("HYDRO_KZ_ZONE")) : 0;
@@ -381,6 +392,7 @@ void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, D
   if (kz_env > 0) {
     kz = std::min(kz_env, nz);
     G = (int)(T.units / nz) * ((nz + kz - 1) / kz);
+    T.zblk = nz;  // the chunked schedule indexes units column-major
   } else {
     G = (int)std::min<int64_t>(slots, T.units);
   }

@@ -62,6 +62,8 @@ struct ZoneTask {
   int32_t slot, tcols;
   int32_t zlo[3], zhi[3];
   int64_t u0, units;
+  int32_t zblk;  // planes per z-block of the unit order (kernel_zone.cu; = planes: column-major)
+  int32_t pad_;
 };
 
 // Initialisation.
