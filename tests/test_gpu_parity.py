@@ -192,3 +192,30 @@ def test_full_size_512_eight_domains_corner_window(path):
     for k in ("u", "v", "w", "e"):
         assert np.abs(far[k]).max() == 0.0, k
     assert np.abs(mid["u"]).max() == 0.0 and np.abs(mid["e"]).max() == 0.0
+
+
+PHYS = [  # readings R5 (gamma 5/3 as a second EOS), R7 (Sedov q coefficients 0.25 / 1.0), R8
+    dict(gamma=5.0 / 3.0),
+    dict(q_lin=0.25, q_quad=1.0),
+    dict(q_lin=0.0, q_quad=0.0),  # no viscosity at all
+    dict(cfl=0.5, c_vol=0.2, dt_growth=1.05),
+    dict(dt_max=2e-4, reflect_mask=0b010101),  # dt cap; walls only on the low faces
+]
+
+
+@pytest.mark.parametrize("path", PATHS)
+@pytest.mark.parametrize("phys", range(len(PHYS)))
+def test_physics_parameters(phys, path):
+    """The C ABI's physics parameters (hydro_config: gamma, q_lin, q_quad, cfl, c_vol, dt_growth,
+    dt_max, reflect_mask) reach every kernel path: jittered 18x16x14 (several tiles, ragged) and
+    Sedov 24^3 in 2 x 2 domains, against the oracle with the same parameters."""
+    n = (18, 16, 14)
+    for kw in (dict(n=n, init="user", user=jittered_state(n, 4), **PHYS[phys]),
+               dict(n=(24, 24, 24), ndom=(2, 2, 1), **PHYS[phys])):
+        for nc, tol in ((1, 1e-12), (60, 1e-10)):
+            fo, io = oracle.run(ocfg(kw), nc)
+            fg, ig = run_gpu(nc, path=path, **kw)
+            assert ig["status"] == io.get("status", 0) == 0, (ig, io)
+            compare(fg, fo, tol)
+            assert ig["dt"] == pytest.approx(io["dt"], rel=tol)
+            assert ig["t"] == pytest.approx(io["t"], rel=tol)
