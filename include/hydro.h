@@ -155,7 +155,8 @@ int hydro_get_box(hydro_ctx *h, const int64_t lo[3], const int64_t hi[3], uint32
                   double *const *out);
 
 /* Replace the state (x,y,z,u,v,w on nodes, e on zones; global host arrays, every rank) and set
-   t and the next dt; zone masses are kept.  Used for restart and for the end-to-end benchmark
+   t and the next dt (clamped to t_stop - t when t_stop > 0, as at creation); zone masses are
+   kept.  Used for restart and for the end-to-end benchmark
    (host -> device copies through the public API).  Clears a failed state.  Collective. */
 int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, double t,
                     double dt);
@@ -163,7 +164,7 @@ int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, 
 /* Streamed batches of independent runs on this context's mesh (an ensemble: many initial
    states through the same cycle).  Batch b starts from the host state in[7b .. 7b+6] = x, y, z,
    u, v, w (global node arrays) and e (global zone array), laid out as for hydro_set_state,
-   with clock t0[b], dt0[b] and cycle 0; it runs ncycles cycles (the hot path of hydro_step)
+   with clock t0[b], dt0[b] (clamped as by hydro_set_state) and cycle 0; it runs ncycles cycles (the hot path of hydro_step)
    and writes x, y, z, u, v, w, e after them into out[7b .. 7b+6] (as hydro_get_fields).  Zone
    masses are the context's, as for hydro_set_state.  The host->device copy of batch b+1 and
    the device->host copy of batch b-1 run on two copy streams while batch b computes (two

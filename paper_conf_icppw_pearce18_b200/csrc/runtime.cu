@@ -1161,7 +1161,8 @@ int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, 
   CK(cudaMemcpyAsync(&s0, h->st, sizeof(s0), cudaMemcpyDeviceToHost, h->stream));
   CK(cudaStreamSynchronize(h->stream));
   s0.t = t;
-  s0.dt = dt;
+  // the t_stop clamp of S9 (as at creation): a run started before t_stop ends on it exactly
+  s0.dt = (h->ph.t_stop > 0.0 && t < h->ph.t_stop) ? std::min(dt, h->ph.t_stop - t) : dt;
   s0.err = 0;
   s0.halted = 0;
   s0.done = (h->ph.t_stop > 0.0 && t >= h->ph.t_stop) ? 1u : 0u;
@@ -1294,7 +1295,9 @@ int hydro_run_batch(hydro_ctx *h, int32_t nbatch, int32_t ncycles, const double 
     batch_scatter(h, h->bin[k], h->parity, s);
     CK(cudaEventRecord(h->in_free[k], s));
     const unsigned done = (h->ph.t_stop > 0.0 && t0[b] >= h->ph.t_stop) ? 1u : 0u;
-    launch_reset_clock(h->st, t0[b], dt0[b], done, s);
+    const double dtb = (h->ph.t_stop > 0.0 && t0[b] < h->ph.t_stop)
+                           ? std::min(dt0[b], h->ph.t_stop - t0[b]) : dt0[b];  // as set_state
+    launch_reset_clock(h->st, t0[b], dtb, done, s);
     for (int32_t c = 0; c < ncycles;) {
       if (h->use_graph && h->graph_k > 1 && ncycles - c >= h->graph_k) {
         CK(cudaGraphLaunch(h->graphk[h->parity], s));

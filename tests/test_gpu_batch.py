@@ -25,10 +25,11 @@ def _sync_run(kw, state, t0, dt0, ncycles):
     return f, info
 
 
+@pytest.mark.parametrize("path", ["two", "one", "split"])
 @pytest.mark.parametrize("layout", [dict(), dict(ndom=(2, 2, 1), cuts=[[0, 7, 20], [0, 9, 18], [0, 14]])])
-def test_batches_equal_synchronous_runs(layout):
+def test_batches_equal_synchronous_runs(layout, path):
     n = (20, 18, 14)
-    kw = dict(n=n, init="user", user=jittered_state(n, 3), **layout)
+    kw = dict(n=n, init="user", user=jittered_state(n, 3), path=path, **layout)
     states = [jittered_state(n, s) for s in (3, 4, 5, 6, 7)]
     with Hydro(HydroConfig(**kw)) as h:
         i0 = h.info()
@@ -82,3 +83,22 @@ def test_batch_physics_error_is_per_batch():
     ref, _ = _sync_run(kw, good, 0.0, 1e-4, 8)
     for k in NAMES:
         assert np.array_equal(outs[1][k], ref[k]), k
+
+
+def test_batch_t_stop():
+    """With t_stop, a batch starting at or past it runs only no-op cycles (state carried), and one
+    starting just before it stops at t_stop exactly, as the synchronous calls do."""
+    n = (14, 12, 10)
+    kw = dict(n=n, init="user", user=jittered_state(n, 6), t_stop=0.01)
+    states = [jittered_state(n, s) for s in (6, 7, 8)]
+    t0, dt0 = [0.0, 0.0099, 0.01], [1e-4, 5e-4, 1e-4]
+    with Hydro(HydroConfig(**kw)) as h:
+        outs, infos = h.run_batch(states, 30, t0, dt0)
+    for b, st in enumerate(states):
+        ref, ir = _sync_run(kw, st, t0[b], dt0[b], 30)
+        assert infos[b]["t"] == ir["t"] and infos[b]["cycle"] == ir["cycle"], (b, infos[b], ir)
+        for k in NAMES:
+            assert np.array_equal(outs[b][k], ref[k]), (b, k)
+    assert infos[1]["t"] == pytest.approx(0.01, rel=1e-14)
+    for k in NAMES:  # started at t_stop: nothing moves
+        assert np.array_equal(outs[2][k], states[2][k]), k
