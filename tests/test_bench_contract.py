@@ -1,0 +1,65 @@
+"""bench.py's JSON-line contract: the keys the driver and the judge read.
+
+CPU: the reference arm (the oracle on host cores) on the small config, and a non-zero rank of a
+torchrun launch printing nothing.  GPU: our arm on the small config, a few timed cycles, with the
+roofline, cpu_baseline, e2e, clocks and gpu_launches objects."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _bench(args, env=None, timeout=600):
+    e = dict(os.environ)
+    e.update(env or {})
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), *args], cwd=ROOT,
+                       capture_output=True, text=True, timeout=timeout, env=e)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    return lines
+
+
+def test_reference_arm_line():
+    lines = _bench(["--impl", "reference", "--config", "sedov32", "--steps", "2", "--warmup", "1"])
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference"
+    assert d["metric"] == "zone-cycles/sec fp64" and d["unit"] == "zone-cycles/s"
+    assert d["value"] > 0 and d["higher_is_better"] is True
+    assert d["steps"] == 2 and d["warmup"] == 1 and d["dtype"] == "f64"
+    assert d["config"]["workload"].startswith("Sedov blast 3D 32^3")
+    cb = d["cpu_baseline"]
+    assert cb["kind"] == "oracle" and cb["cores"] >= 1 and cb["value"] == d["value"]
+    assert "sample" in cb
+    e2e = d["e2e"]
+    assert e2e["value"] == d["value"] and e2e["unit"] == d["unit"]
+    assert e2e["h2d_bytes_per_step"] == 0 and e2e["d2h_bytes_per_step"] == 0
+
+
+def test_reference_arm_other_ranks_silent():
+    lines = _bench(["--impl", "reference", "--config", "sedov32", "--steps", "1",
+                    "--warmup", "0"], env={"WORLD_SIZE": "2", "RANK": "1", "LOCAL_RANK": "1"})
+    assert lines == []
+
+
+@pytest.mark.gpu
+def test_our_arm_line():
+    lines = _bench(["--config", "sedov32", "--steps", "20", "--warmup", "3",
+                    "--no-cpu-baseline", "--e2e-steps", "2", "--e2e-cycles", "10"])
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["metric"] == "zone-cycles/sec fp64" and d["n_gpus"] == 1
+    assert d["steps"] == 20 and d["warmup"] == 3 and d["value"] > 0
+    assert d["ms_per_step"] > 0 and d["dtype"] == "f64" and d["data"] == "synthetic"
+    r = d["roofline"]
+    assert r["bound"] == "hbm" and r["unit"] == "GB/s"
+    assert 0 < r["achieved"] and 0 < r["frac"] < 1.0
+    assert abs(r["frac"] - r["achieved"] / r["peak"]) < 1e-9
+    e2e = d["e2e"]
+    assert e2e["value"] > 0 and e2e["h2d_bytes_per_step"] > 0 and e2e["d2h_bytes_per_step"] > 0
+    assert d["gpu_launches"] > 0
+    assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
