@@ -217,7 +217,10 @@ def run_reference(args):
     o.close()
     v = sz * args.steps / el
     line = {"metric": METRIC, "value": v, "unit": "zone-cycles/s", "impl": "reference",
-            "n_gpus": 0, "steps": args.steps, "warmup": args.warmup,
+            # n_gpus: the N of this launch (the driver pairs the arms by N); the oracle itself
+            # runs on rank 0's host cores only, as cpu_baseline / "device" say
+            "n_gpus": max(ws, args.gpus), "device": "host cpu (oracle, rank 0 only)",
+            "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1e3 * el / args.steps, "higher_is_better": True, "scaling": scaling,
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": desc, "sample": list(sample_n)},

@@ -31,6 +31,7 @@ def test_reference_arm_line():
     assert d["metric"] == "zone-cycles/sec fp64" and d["unit"] == "zone-cycles/s"
     assert d["value"] > 0 and d["higher_is_better"] is True
     assert d["steps"] == 2 and d["warmup"] == 1 and d["dtype"] == "f64"
+    assert d["n_gpus"] == 1 and d["device"].startswith("host cpu")
     assert d["config"]["workload"].startswith("Sedov blast 3D 32^3")
     cb = d["cpu_baseline"]
     assert cb["kind"] == "oracle" and cb["cores"] >= 1 and cb["value"] == d["value"]
