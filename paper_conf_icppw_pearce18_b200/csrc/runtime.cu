@@ -336,7 +336,8 @@ int upload_state(hydro_ctx *h, int par, const double *const *nodes6, const doubl
 // S9 can run inside the cycle's last kernel when that kernel is the only one of the cycle (one
 // domain, one rank, not the plain split path).  Measured on B200 at 128^3 it is slower (the
 // per-CTA __threadfence before the ticket delays every CTA's exit: node stage 106 -> 110 us,
-// while a separate k_finalize costs ~2.6 us), so it is off unless built with -DHYDRO_FOLD.
+// while a separate k_finalize costs ~2.6 us; re-measured with the current node stage
+// (tools/gp_fold.sh): 140.4 vs 139.1 us per cycle), so it is off unless built with -DHYDRO_FOLD.
 int fold_finalize(const hydro_ctx *h) {
 #ifndef HYDRO_FOLD
   (void)h;
