@@ -35,7 +35,7 @@
 extern "C" {
 #endif
 
-#define HYDRO_ABI_VERSION 2
+#define HYDRO_ABI_VERSION 3
 
 typedef struct hydro_ctx hydro_ctx; /* opaque; owned by the library */
 
@@ -47,7 +47,8 @@ enum {
   HYDRO_ENCCL = -4,      /* communicator error */
   HYDRO_ETANGLED = -5,   /* a zone volume became <= 0 */
   HYDRO_ENONFINITE = -6, /* a non-finite pressure or dt appeared */
-  HYDRO_EDTMIN = -7,     /* reserved: dt fell below a floor */
+  HYDRO_EDTMIN = -7,     /* the zone dt minimum of a cycle fell below hydro_config.dt_floor
+                            (dt collapse, reading R23; bad_zone = -1: a global condition) */
   HYDRO_ESTATE = -8      /* the context failed earlier; only get_fields/destroy still work */
 };
 
@@ -111,6 +112,11 @@ typedef struct {
                                    (Flanagan-Belytschko).  0 = off (the default,
                                    north_star's phase list).  kappa > 0 runs the split kernels
                                    (corner-force planes in HBM), whatever the path flags say. */
+  double dt_floor;              /* dt-collapse floor (reading R23): > 0 absolute;
+                                   0 (the default) = 1e-6 * dt^0 (dt^0 before the t_stop clamp);
+                                   < 0 = no floor.  A cycle whose min_z dt_z falls below it halts
+                                   the run with HYDRO_EDTMIN (state = the one after that cycle),
+                                   unless that cycle reaches t_stop. */
 } hydro_config;
 
 typedef struct {
@@ -124,7 +130,7 @@ typedef struct {
 
 /* Fill cfg with the defaults of DESIGN.md §3 (gamma 1.4, q 0.5/2.0, cfl 0.3, c_vol 0.1,
    dt_growth 1.1, dt_max = dt_init = +inf, reflecting walls, Sedov on [0,1.2]^3 with
-   sedov_energy = 0.851072/8, single rank, device 0). */
+   sedov_energy = 0.851072/8, dt_floor 0 = 1e-6 dt^0, single rank, device 0). */
 void hydro_config_default(hydro_config *cfg);
 
 /* Create: validate cfg, build the layout (domains, halo maps, domain->rank map), allocate the
@@ -186,7 +192,15 @@ int hydro_run_batch(hydro_ctx *h, int32_t nbatch, int32_t ncycles, const double 
 int hydro_peer_export(hydro_ctx *h, void *buf, size_t *len);
 int hydro_peer_import(hydro_ctx *h, const void *all, size_t len_per_rank);
 
-/* Current info without stepping. */
+/* Peer transport teardown, step 1 of 3 (collective order): close this rank's mappings of the
+   other ranks' memory after its own work drained.  Then the caller barriers over all ranks, then
+   every rank calls hydro_destroy (which frees memory the others had mapped: freeing it while
+   another process still has it open is undefined in CUDA).  No-op without HYDRO_FLAG_PEER.
+   After it, hydro_step returns HYDRO_ESTATE. */
+int hydro_peer_detach(hydro_ctx *h);
+
+/* Current info without stepping.  Local (not a collective): the status is already identical on
+   every rank because both transports OR-reduce the error bits with dt every cycle. */
 int hydro_get_info(hydro_ctx *h, hydro_info *info);
 
 /* Domain migration: the complete state of one domain this rank owns, i.e.
@@ -196,9 +210,12 @@ int hydro_get_info(hydro_ctx *h, hydro_info *info);
    storage depends only on the domain box, so a buffer packed by one context unpacks into any
    context with the same cuts, on any rank; moving it between ranks is the caller's (e.g.
    torch.distributed send/recv over NCCL).  hydro_domain_bytes: *len = bytes of dom's buffer
-   (host-only arithmetic, any domain).  pack: dev_buf (device, >= len bytes, caller-owned)
-   <- state, on `stream` (NULL = the context's), synchronised before return.  unpack: state <-
-   dev_buf, then 1/m and the nodal 8/sum m are recomputed for that domain.  Errors:
+   (host-only arithmetic, any domain).  pack: dev_buf (device memory, or host memory: the
+   copies use the unified address space, page-locked host memory runs at DMA speed; >= len
+   bytes, caller-owned) <- state, on `stream` (NULL = the context's), synchronised before
+   return.  unpack: state <- dev_buf (same), then 1/m and the nodal 8/sum m are recomputed for
+   that domain.  With host buffers this pair is the rank-local end-to-end path (bench.py e2e at
+   N > 1: each rank moves exactly its own domains).  Errors:
    HYDRO_EINVAL (dom not owned by this rank, len too small), HYDRO_ECUDA. */
 int hydro_domain_bytes(const hydro_ctx *h, int32_t dom, size_t *len);
 int hydro_domain_pack(hydro_ctx *h, int32_t dom, void *dev_buf, size_t len, void *stream);

@@ -72,6 +72,7 @@ class _Config(C.Structure):
         ("rho0", C.c_double), ("e0", C.c_double), ("sedov_energy", C.c_double),
         ("user", C.POINTER(C.c_double) * 8),
         ("hg_coef", C.c_double),
+        ("dt_floor", C.c_double),
     ]
 
 
@@ -109,6 +110,7 @@ class OracleConfig:
     sedov_energy: float = 0.851072 / 8.0   # reading R10: octant share, R(t=1)=1 for gamma=1.4
     user: Optional[Dict[str, np.ndarray]] = None
     hg_coef: float = 0.0                  # reading R17 / SURVEY §8f f1: hourglass kappa, 0 = off
+    dt_floor: float = 0.0                 # reading R23: > 0 absolute, 0 = 1e-6 dt^0, < 0 none
 
 
 class OracleError(RuntimeError):
@@ -136,7 +138,8 @@ class Oracle:
                 self._keep.append(arr)
                 c.cuts[a] = arr.ctypes.data_as(C.POINTER(C.c_int64))
         for k in ("gamma", "q_lin", "q_quad", "cfl", "c_vol", "dt_growth", "dt_max", "dt_init",
-                  "t_stop", "dt_first", "t0", "rho0", "e0", "sedov_energy", "hg_coef"):
+                  "t_stop", "dt_first", "t0", "rho0", "e0", "sedov_energy", "hg_coef",
+                  "dt_floor"):
             setattr(c, k, float(getattr(cfg, k)))
         c.reflect_mask = int(cfg.reflect_mask)
         c.init_kind = INIT[cfg.init]

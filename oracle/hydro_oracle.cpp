@@ -248,6 +248,7 @@ struct orc_ctx {
   int ndx, ndy, ndz;
   std::vector<int32_t> zown[3], nown[3];  // per axis: owning domain coordinate (lowest)
   double t, dt, dtzmin;
+  double dt_floor;  // reading R23: 0 = none
   int64_t cycle;
   int failed;
   int64_t bad_zone;
@@ -522,8 +523,11 @@ void cycle(orc_ctx *h) {
   h->dtzmin = dtmin;
   h->dt = dtn;
   h->cycle += 1;
-  if (!(std::isfinite(dtn) && dtn > 0.0) && !(c.t_stop > 0.0 && tn >= c.t_stop))
-    fail(h, ORC_ENONFINITE, -1);
+  const bool stop = c.t_stop > 0.0 && tn >= c.t_stop;
+  if (!(std::isfinite(dtn) && dtn > 0.0) && !stop) fail(h, ORC_ENONFINITE, -1);
+  // Reading R23: dt collapse.  The zone dt minimum of this cycle fell below the floor: the run
+  // halts (state = the one after this cycle), a global condition, so no bad zone is named.
+  if (!stop && dtmin < h->dt_floor) fail(h, ORC_EDTMIN, -1);
 }
 
 bool valid_config(const orc_config *c) {
@@ -650,6 +654,9 @@ int orc_create(const orc_config *cfg, orc_ctx **out) {
   h->dtzmin = dtmin;
   h->dt = (cfg->dt_first > 0.0) ? cfg->dt_first
                                  : std::min(std::min(cfg->dt_init, cfg->dt_max), dtmin);
+  // reading R23: the floor is relative to dt^0 (before the t_stop clamp) unless given
+  h->dt_floor = cfg->dt_floor > 0.0 ? cfg->dt_floor
+                : (cfg->dt_floor == 0.0 && std::isfinite(h->dt)) ? 1e-6 * h->dt : 0.0;
   if (cfg->t_stop > 0.0) h->dt = std::min(h->dt, cfg->t_stop - h->t);
   if (h->failed) {
     const int code = h->failed;

@@ -31,6 +31,7 @@ enum {
   ORC_EINVAL = -1,
   ORC_ETANGLED = -5,   /* a zone volume <= 0 */
   ORC_ENONFINITE = -6, /* non-finite P or dt */
+  ORC_EDTMIN = -7,     /* min_z dt_z of a cycle fell below the dt floor (reading R23) */
   ORC_ESTATE = -8      /* context already failed */
 };
 
@@ -50,6 +51,9 @@ typedef struct {
      [6] = rho (USER) or zone mass (USER_MASS) on n^3 zones; [7] = e on zones. */
   const double *user[8];
   double hg_coef;               /* viscous hourglass coefficient kappa >= 0 (reading R17; 0 = off) */
+  double dt_floor;              /* dt-collapse floor (reading R23): > 0 absolute; 0 = 1e-6 * dt^0;
+                                   < 0 = none.  A cycle whose min_z dt_z is below it halts the run
+                                   with ORC_EDTMIN (bad_zone -1), unless it ends the run at t_stop */
 } orc_config;
 
 typedef struct {

@@ -1,7 +1,9 @@
 // comm.cu -- see comm.h.  NCCL transport for ranks > 1.
 #include <nccl.h>
 
+#include <chrono>
 #include <cstring>
+#include <thread>
 
 #include "comm.h"
 
@@ -47,6 +49,20 @@ __global__ void k_pack(const DomView *views, const SlabDesc *descs, double *buf,
   }
 }
 
+// dt / error words for the allreduce (see comm.h): red[0] = ~dt bits, red[1 + b] = error bit b
+__global__ void k_red_pack(const DevState *st, unsigned long long *red) {
+  red[0] = ~st->dtz_acc;
+#pragma unroll
+  for (int b = 0; b < 3; ++b) red[1 + b] = (st->err >> b) & 1u;
+}
+__global__ void k_red_unpack(DevState *st, const unsigned long long *red) {
+  st->dtz_acc = ~red[0];
+  unsigned e = 0;
+#pragma unroll
+  for (int b = 0; b < 3; ++b) e |= red[1 + b] ? (1u << b) : 0u;
+  st->err = e;
+}
+
 }  // namespace
 
 struct Comm {
@@ -57,7 +73,7 @@ struct Comm {
   double *sendbuf = nullptr, *recvbuf = nullptr;
   int64_t send_total = 0, recv_total = 0;
   DomView *views_dev[2] = {nullptr, nullptr};
-  int *status_dev = nullptr;
+  unsigned long long *red_dev = nullptr;  // [4]: the S9 allreduce words
 };
 
 int comm_unique_id(void *out128) {
@@ -114,7 +130,7 @@ int comm_create(Comm **out, const hydro_config *cfg, const Layout &L,
     if (e != cudaSuccess) *err = cudaGetErrorString(e);
     return e == cudaSuccess;
   };
-  if (!ck(cudaMalloc(&c->status_dev, sizeof(int)))) return HYDRO_ECUDA;
+  if (!ck(cudaMalloc(&c->red_dev, 4 * sizeof(unsigned long long)))) return HYDRO_ECUDA;
   if (c->send_total) {
     if (!ck(cudaMalloc(&c->sendbuf, c->send_total * sizeof(double)))) return HYDRO_ENOMEM;
     if (!ck(cudaMalloc(&c->sends_dev, c->sends.size() * sizeof(SlabDesc)))) return HYDRO_ENOMEM;
@@ -150,10 +166,12 @@ int comm_bind_views(Comm *c, const DomView *const *v0, const DomView *const *v1,
   return HYDRO_OK;
 }
 
-int comm_dt_min(Comm *c, unsigned long long *dev_bits, cudaStream_t s) {
-  if (ncclAllReduce(dev_bits, dev_bits, 1, ncclUint64, ncclMin, c->nccl, s) != ncclSuccess)
+int comm_dt_min(Comm *c, DevState *st, cudaStream_t s) {
+  k_red_pack<<<1, 1, 0, s>>>(st, c->red_dev);
+  if (ncclAllReduce(c->red_dev, c->red_dev, 4, ncclUint64, ncclMax, c->nccl, s) != ncclSuccess)
     return HYDRO_ENCCL;
-  return HYDRO_OK;
+  k_red_unpack<<<1, 1, 0, s>>>(st, c->red_dev);
+  return cudaGetLastError() == cudaSuccess ? HYDRO_OK : HYDRO_ECUDA;
 }
 
 int comm_halo(Comm *c, int par, cudaStream_t s) {
@@ -176,18 +194,37 @@ int comm_halo(Comm *c, int par, cudaStream_t s) {
   return cudaGetLastError() == cudaSuccess ? HYDRO_OK : HYDRO_ECUDA;
 }
 
-int comm_status_agree(Comm *c, int status) {
-  int v = status;
-  cudaMemcpy(c->status_dev, &v, sizeof(int), cudaMemcpyHostToDevice);
-  if (ncclAllReduce(c->status_dev, c->status_dev, 1, ncclInt32, ncclMin, c->nccl, 0) !=
-      ncclSuccess)
-    return HYDRO_ENCCL;
-  cudaMemcpy(&v, c->status_dev, sizeof(int), cudaMemcpyDeviceToHost);
-  return v;
+int comm_wait(Comm *c, cudaStream_t s, double timeout_s, std::string *err) {
+  if (!c->nccl) return HYDRO_OK;  // aborted earlier: the caller's stream sync reports the rest
+  const auto t0 = std::chrono::steady_clock::now();
+  for (int spin = 0;; ++spin) {
+    const cudaError_t q = cudaStreamQuery(s);
+    if (q == cudaSuccess) return HYDRO_OK;
+    if (q != cudaErrorNotReady) {
+      *err = std::string("stream: ") + cudaGetErrorString(q);
+      return HYDRO_ECUDA;
+    }
+    ncclResult_t ae = ncclSuccess;
+    if (ncclCommGetAsyncError(c->nccl, &ae) != ncclSuccess || ae != ncclSuccess) {
+      *err = std::string("NCCL asynchronous error: ") + ncclGetErrorString(ae);
+      ncclCommAbort(c->nccl);
+      c->nccl = nullptr;
+      return HYDRO_ENCCL;
+    }
+    const double el =
+        std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    if (timeout_s > 0.0 && el > timeout_s) {
+      *err = "NCCL wait timed out (a peer rank stalled or died)";
+      ncclCommAbort(c->nccl);
+      c->nccl = nullptr;
+      return HYDRO_ENCCL;
+    }
+    if (spin > 64) std::this_thread::sleep_for(std::chrono::microseconds(50));
+  }
 }
 
 int comm_kernels_per_cycle(const Comm *c) {
-  return (c->sends.empty() ? 0 : 1) + (c->recvs.empty() ? 0 : 1);
+  return (c->sends.empty() ? 0 : 1) + (c->recvs.empty() ? 0 : 1) + 2;  // + dt pack/unpack
 }
 
 void comm_destroy(Comm *c) {
@@ -199,7 +236,7 @@ void comm_destroy(Comm *c) {
   cudaFree(c->recvs_dev);
   cudaFree(c->views_dev[0]);
   cudaFree(c->views_dev[1]);
-  cudaFree(c->status_dev);
+  cudaFree(c->red_dev);
   delete c;
 }
 

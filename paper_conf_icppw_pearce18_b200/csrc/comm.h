@@ -2,8 +2,10 @@
 // exchange with neighbouring domains on other ranks ("halo exchange" between
 // neighbouring domains; L513-520: the paper routed it through the host, GPU-direct was future
 // work) and the global dt min-reduction (S9).  Transport: NCCL 2.28 over NVLink/NVSwitch,
-// grouped ncclSend/ncclRecv for the halo, ncclAllReduce(min, uint64) on the bit pattern of the
-// non-negative dt (bit order == numeric order for non-negative doubles).
+// grouped ncclSend/ncclRecv for the halo, and one ncclAllReduce(max, uint64) per cycle over
+// [~dt bits, one word per error bit]: the complemented bit pattern of the non-negative dt gives
+// the min (bit order == numeric order for non-negative doubles), the error words give the OR,
+// so every rank latches the same status (a tangled zone on one rank halts all of them).
 #pragma once
 #include <cuda_runtime.h>
 
@@ -25,12 +27,14 @@ int comm_create(Comm **out, const hydro_config *cfg, const Layout &L,
 // views_p[slot] = &DomView of parity p for every local domain slot (kept by pointer).
 int comm_bind_views(Comm *c, const DomView *const *views0, const DomView *const *views1, int n,
                     std::string *err);
-// In-place global min of a device uint64 (dt bits).
-int comm_dt_min(Comm *c, unsigned long long *dev_bits, cudaStream_t s);
+// Global S9 inputs: st->dtz_acc <- min over ranks, st->err <- OR over ranks (in place, on s).
+int comm_dt_min(Comm *c, DevState *st, cudaStream_t s);
 // Exchange the next-parity ghost slabs of parity-`par` views with remote neighbours.
 int comm_halo(Comm *c, int par, cudaStream_t s);
-// Agree on a status code across ranks (the most negative wins).
-int comm_status_agree(Comm *c, int status);
+// Wait for stream s while polling the communicator: returns HYDRO_OK once s is
+// idle, HYDRO_ENCCL (after ncclCommAbort) on an asynchronous NCCL error or when the wait exceeds
+// timeout_s seconds (a peer that died or a mismatched plan would otherwise hang the caller).
+int comm_wait(Comm *c, cudaStream_t s, double timeout_s, std::string *err);
 int comm_kernels_per_cycle(const Comm *c);
 void comm_destroy(Comm *c);
 

@@ -63,12 +63,13 @@ struct DevState {
   unsigned int done;            // t >= t_stop
   unsigned int blocks_done;     // CTAs of the last cycle kernel that finished (folded finalize)
   unsigned long long xchg;      // peer-transport exchange epoch (peer.cu)
+  double dt_floor;              // reading R23: min_z dt_z below this halts the run (0 = none)
 };
 
-enum : unsigned int { ERR_TANGLED = 1u, ERR_NONFINITE = 2u };
+enum : unsigned int { ERR_TANGLED = 1u, ERR_NONFINITE = 2u, ERR_DTMIN = 4u };
 
 // S9: t' = t + dt, dt' = min(min(growth*dt, dt_max), min_z dt_z), t_stop clamp;
-// latch the cycle's error bits so later cycles become no-ops (the state stays the one after the
+// dt-collapse check (reading R23); latch the cycle's error bits so later cycles become no-ops (the state stays the one after the
 // failing cycle, as in the oracle).  Run by one thread after every kernel of the cycle.
 // PDL (kernels.h launch_pdl): wait for the preceding kernel's completion and memory flush, then
 // let the next kernel launch.  No-ops when the kernel was launched without the attribute.
@@ -92,6 +93,8 @@ __device__ __forceinline__ void finalize_cycle(DevState *st, const Phys &ph) {
   st->dtz_acc = (unsigned long long)__double_as_longlong(INFINITY);
   unsigned err = st->err;
   if (!(isfinite(dtn) && dtn > 0.0) && !stop) err |= ERR_NONFINITE;
+  // reading R23: dt collapse (the zone dt minimum of this cycle fell below the floor)
+  if (!stop && dtmin < st->dt_floor) err |= ERR_DTMIN;
   st->halted = err;
   st->done = stop ? 1u : 0u;
 }

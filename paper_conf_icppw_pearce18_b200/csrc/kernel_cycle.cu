@@ -715,9 +715,17 @@ int choose_kz(int tiles, int n2, int sms) {
   return std::min(best, n2);
 }
 
+// The shared-memory opt-in is a per-device function attribute: cached per device ordinal.
+int cur_device() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  return dev < 0 ? 0 : (dev >= 64 ? 63 : dev);
+}
+
 template <bool FUSED, int TY>
 void set_smem() {
-  static bool done = false;
+  static bool done_dev[64] = {};
+  bool &done = done_dev[cur_device()];
   if (!done) {
     using T = CTile<CTX, TY>;
     cudaFuncSetAttribute(k_cycle<CTX, TY, FUSED, false>,
@@ -730,12 +738,10 @@ void set_smem() {
 }
 
 int num_sms() {
-  static int sms = 0;
-  if (!sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  }
+  static int sms_dev[64] = {};
+  const int dev = cur_device();
+  int &sms = sms_dev[dev];
+  if (!sms) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   return sms;
 }
 

@@ -361,11 +361,13 @@ ZoneTask zone_task(const DomView &d, int slot) {
   return T;
 }
 
-int zone_slots() {
-  static int slots = 0;
+int zone_slots() {  // per device: the shared-memory opt-in is a per-device attribute
+  static int slots_dev[64] = {};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int &slots = slots_dev[dev < 0 ? 0 : (dev >= 64 ? 63 : dev)];
   if (!slots) {
-    int dev = 0, sms = 0, per_sm = 0;
-    cudaGetDevice(&dev);
+    int sms = 0, per_sm = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     for (auto k : {k_zone_stage<false>, k_zone_stage<true>})
       cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ZBYTES);

@@ -80,7 +80,7 @@ void launch_nodal_mass(const DomView &d, cudaStream_t s);
 // dt^0 (S2-S6 at x^0 with no predictor) over owned zones -> st->dtz_acc, error flags.
 void launch_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 void launch_finalize_init(DevState *st, double dt_first, double dt_init, double dt_max,
-                          double t_stop, double t0, cudaStream_t s);
+                          double t_stop, double t0, double dt_floor, cudaStream_t s);
 
 // Split 3-kernel pipeline (naive, obviously-correct path; HYDRO_FLAG_SPLIT).
 void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);

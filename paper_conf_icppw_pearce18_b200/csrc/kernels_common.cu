@@ -137,9 +137,11 @@ __global__ void k_dt0(DomView d, Phys ph, DevState *st) {
 }
 
 __global__ void k_finalize_init(DevState *st, double dt_first, double dt_init, double dt_max,
-                                double t_stop, double t0) {
+                                double t_stop, double t0, double dt_floor) {
   const double dtmin = __longlong_as_double((long long)st->dtz_acc);
   double dt = dt_first > 0.0 ? dt_first : fmin(fmin(dt_init, dt_max), dtmin);
+  // reading R23: the dt-collapse floor, relative to dt^0 (before the t_stop clamp) unless given
+  st->dt_floor = dt_floor > 0.0 ? dt_floor : (dt_floor == 0.0 && isfinite(dt)) ? 1e-6 * dt : 0.0;
   if (t_stop > 0.0) dt = fmin(dt, t_stop - t0);
   st->t = t0;
   st->dt = dt;
@@ -374,8 +376,8 @@ void launch_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) 
   k_dt0<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph, st);
 }
 void launch_finalize_init(DevState *st, double dt_first, double dt_init, double dt_max,
-                          double t_stop, double t0, cudaStream_t s) {
-  k_finalize_init<<<1, 1, 0, s>>>(st, dt_first, dt_init, dt_max, t_stop, t0);
+                          double t_stop, double t0, double dt_floor, cudaStream_t s) {
+  k_finalize_init<<<1, 1, 0, s>>>(st, dt_first, dt_init, dt_max, t_stop, t0, dt_floor);
 }
 // hydro_run_batch: a fresh clock for the next batch (t, dt given; cycle 0; errors cleared).
 __global__ void k_reset_clock(DevState *st, double t, double dt, unsigned done) {

@@ -300,9 +300,16 @@ void peer_push_targets(const Peer *p, std::vector<PushTarget> *out) {
   out->insert(out->end(), p->targets.begin(), p->targets.end());
 }
 
-void peer_destroy(Peer *p) {
+void peer_detach(Peer *p) {
   if (!p) return;
   for (void *ptr : p->opened) cudaIpcCloseMemHandle(ptr);
+  p->opened.clear();
+  p->ready = false;  // the remote slabs are gone: no more cycles
+}
+
+void peer_destroy(Peer *p) {
+  if (!p) return;
+  peer_detach(p);
   cudaFree(p->mailbox);
   cudaFree(p->mbox_dev);
   cudaFree(p->remote_dev[0]);

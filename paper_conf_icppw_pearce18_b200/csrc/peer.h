@@ -43,6 +43,10 @@ int peer_exchange(Peer *p, const DomView *local_views_dev, int par, bool halo, D
 int peer_kernels_per_cycle(const Peer *p, bool halo);
 // The inter-rank slabs this rank pushes (after peer_import), for the fused-halo tables.
 void peer_push_targets(const Peer *p, std::vector<PushTarget> *out);
+// Close every imported IPC mapping (idempotent).  Teardown order across ranks: every rank
+// detaches, the caller barriers, then every rank frees (CUDA: freeing an allocation another
+// process still has open is undefined).
+void peer_detach(Peer *p);
 void peer_destroy(Peer *p);
 
 }  // namespace hydro

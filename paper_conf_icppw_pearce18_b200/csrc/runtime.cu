@@ -488,7 +488,7 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
   }
   if (h->split) {
     if (h->comm) {
-      int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
+      int rc = comm_dt_min(h->comm, h->st, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
     }
     for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
@@ -496,13 +496,13 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
   } else if (h->one_kernel) {
     for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
     if (h->comm) {
-      int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
+      int rc = comm_dt_min(h->comm, h->st, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
     }
   } else {
     launch_zone_stages(h, par, s);
     if (h->comm) {
-      int rc = comm_dt_min(h->comm, &h->st->dtz_acc, s);
+      int rc = comm_dt_min(h->comm, h->st, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
     }
     launch_node_stages(h, par, s, h->halo_overlap);
@@ -549,14 +549,22 @@ int build_graphs(hydro_ctx *h) {
   return HYDRO_OK;
 }
 
+// Device state -> info.  The status is already identical on every rank (the error bits are
+// OR-reduced with dt every cycle by both transports), so this is not a collective.
 int read_info(hydro_ctx *h, hydro_info *info, cudaStream_t s) {
   DevState st;
   CK(cudaMemcpyAsync(&st, h->st, sizeof(st), cudaMemcpyDeviceToHost, s));
+  if (h->comm) {  // poll NCCL while the cycles drain (HYDRO_NCCL_TIMEOUT_S, default 600 s)
+    static const double tmo =
+        getenv("HYDRO_NCCL_TIMEOUT_S") ? atof(getenv("HYDRO_NCCL_TIMEOUT_S")) : 600.0;
+    int rc = comm_wait(h->comm, s, tmo, &h->err);
+    if (rc) return set_err(h, rc, h->err);
+  }
   CK(cudaStreamSynchronize(s));
   int status = HYDRO_OK;
   if (st.halted & ERR_TANGLED) status = HYDRO_ETANGLED;
   else if (st.halted & ERR_NONFINITE) status = HYDRO_ENONFINITE;
-  if (h->comm) status = comm_status_agree(h->comm, status);
+  else if (st.halted & ERR_DTMIN) status = HYDRO_EDTMIN;
   if (info) {
     info->t = st.t;
     info->dt = st.dt;
@@ -570,7 +578,7 @@ int read_info(hydro_ctx *h, hydro_info *info, cudaStream_t s) {
 
 bool valid_phys(const hydro_config *c) {
   return c->gamma > 1.0 && c->q_lin >= 0.0 && c->q_quad >= 0.0 && c->cfl > 0.0 &&
-         c->c_vol > 0.0 && c->dt_growth > 0.0 && c->dt_max > 0.0 &&
+         c->c_vol > 0.0 && c->dt_growth > 0.0 && c->dt_max > 0.0 && !std::isnan(c->dt_floor) &&
          std::isfinite(c->origin[0]) && c->extent[0] > 0.0 && c->extent[1] > 0.0 &&
          c->extent[2] > 0.0 && c->hg_coef >= 0.0 && std::isfinite(c->hg_coef);
 }
@@ -896,12 +904,12 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
          for (LocalDom &D : h->doms) launch_nodal_mass(D.view[0], h->stream);
          for (LocalDom &D : h->doms) launch_dt0(D.view[0], h->ph, h->st, h->stream);
          if (h->comm) {
-           int r = comm_dt_min(h->comm, &h->st->dtz_acc, h->stream);
+           int r = comm_dt_min(h->comm, h->st, h->stream);
            if (r) return set_err(h, r, "dt allreduce failed");
          }
          if (!h->peer)  // peer transport: dt^0 is reduced over the ranks at hydro_peer_import
            launch_finalize_init(h->st, cfg->dt_first, cfg->dt_init, cfg->dt_max, cfg->t_stop,
-                                cfg->t0, h->stream);
+                                cfg->t0, cfg->dt_floor, h->stream);
          CK(cudaGetLastError());
          CK(cudaStreamSynchronize(h->stream));
          return HYDRO_OK;
@@ -945,7 +953,7 @@ int hydro_peer_import(hydro_ctx *h, const void *all, size_t len_per_rank) {
   rc = peer_exchange(h->peer, h->views_dev[0], 0, false, h->st, h->stream);
   if (rc) return set_err(h, rc, "peer dt^0 exchange failed");
   launch_finalize_init(h->st, h->cfg.dt_first, h->cfg.dt_init, h->cfg.dt_max, h->cfg.t_stop,
-                       h->cfg.t0, h->stream);
+                       h->cfg.t0, h->cfg.dt_floor, h->stream);
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(h->stream));
   if (h->use_graph && (rc = build_graphs(h)) != HYDRO_OK) return rc;
@@ -1018,11 +1026,11 @@ int hydro_domain_pack(hydro_ctx *h, int32_t dom, void *dev_buf, size_t len, void
   char *dst = (char *)dev_buf;
   // the six current node arrays are consecutive allocations of pitch nb (carve_views)
   CK(cudaMemcpy2DAsync(dst, nn * sizeof(double), v.x, nb, nn * sizeof(double), 6,
-                       cudaMemcpyDeviceToDevice, s));
+                       cudaMemcpyDefault, s));
   dst += 6 * nn * sizeof(double);
-  CK(cudaMemcpyAsync(dst, v.e, nz * sizeof(double), cudaMemcpyDeviceToDevice, s));
+  CK(cudaMemcpyAsync(dst, v.e, nz * sizeof(double), cudaMemcpyDefault, s));
   dst += nz * sizeof(double);
-  CK(cudaMemcpyAsync(dst, v.m, nz * sizeof(double), cudaMemcpyDeviceToDevice, s));
+  CK(cudaMemcpyAsync(dst, v.m, nz * sizeof(double), cudaMemcpyDefault, s));
   CK(cudaStreamSynchronize(s));
   return HYDRO_OK;
 }
@@ -1042,11 +1050,11 @@ int hydro_domain_unpack(hydro_ctx *h, int32_t dom, const void *dev_buf, size_t l
   const size_t nb = align_up(nn * sizeof(double), 256);
   const char *src = (const char *)dev_buf;
   CK(cudaMemcpy2DAsync(const_cast<double *>(v.x), nb, src, nn * sizeof(double), nn * sizeof(double), 6,
-                       cudaMemcpyDeviceToDevice, s));
+                       cudaMemcpyDefault, s));
   src += 6 * nn * sizeof(double);
-  CK(cudaMemcpyAsync(const_cast<double *>(v.e), src, nz * sizeof(double), cudaMemcpyDeviceToDevice, s));
+  CK(cudaMemcpyAsync(const_cast<double *>(v.e), src, nz * sizeof(double), cudaMemcpyDefault, s));
   src += nz * sizeof(double);
-  CK(cudaMemcpyAsync(const_cast<double *>(v.m), src, nz * sizeof(double), cudaMemcpyDeviceToDevice, s));
+  CK(cudaMemcpyAsync(const_cast<double *>(v.m), src, nz * sizeof(double), cudaMemcpyDefault, s));
   launch_nodal_mass(D.view[0], s);  // 1/m and 8 / sum m from the imported masses
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(s));
@@ -1389,15 +1397,15 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
     CK(cudaEventRecord(ev[4], s));
     if (h->split) {
       for (LocalDom &D : h->doms) launch_zone_split(D.view[par], h->ph, h->st, s);
-      if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
+      if (h->comm && comm_dt_min(h->comm, h->st, s)) return HYDRO_ENCCL;
       for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
       for (LocalDom &D : h->doms) launch_energy_split(D.view[par], h->ph, h->st, s);
     } else if (h->one_kernel) {
       for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
-      if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
+      if (h->comm && comm_dt_min(h->comm, h->st, s)) return HYDRO_ENCCL;
     } else {
       launch_zone_stages(h, par, s);
-      if (h->comm && comm_dt_min(h->comm, &h->st->dtz_acc, s)) return HYDRO_ENCCL;
+      if (h->comm && comm_dt_min(h->comm, h->st, s)) return HYDRO_ENCCL;
       CK(cudaEventRecord(ev[4], s));
       launch_node_stages(h, par, s);
     }
@@ -1438,6 +1446,16 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
   const int status = read_info(h, &info, s);
   if (status < 0 && status != HYDRO_ECUDA) h->failed = status;
   return status;
+}
+
+int hydro_peer_detach(hydro_ctx *h) {
+  if (!h) return HYDRO_OK;
+  if (!h->peer) return HYDRO_OK;
+  CK(cudaSetDevice(h->device));
+  CK(cudaStreamSynchronize(h->stream));
+  CK(cudaDeviceSynchronize());  // no cycle of this rank still stores into a peer
+  peer_detach(h->peer);
+  return HYDRO_OK;
 }
 
 int hydro_destroy(hydro_ctx *h) {

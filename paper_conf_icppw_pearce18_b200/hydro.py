@@ -22,7 +22,7 @@ LIB_PATH = os.environ.get("HYDRO_LIB") or os.path.join(_HERE, "libhydro_b200.so"
 NODE_FIELDS = ("x", "y", "z", "u", "v", "w")
 ZONE_FIELDS = ("rho", "e", "p", "q", "c", "vol", "mass")
 ALL_FIELDS = NODE_FIELDS + ZONE_FIELDS
-ABI_VERSION = 2
+ABI_VERSION = 3
 FLAG_NO_GRAPH = 1 << 0
 FLAG_SPLIT = 1 << 1
 FLAG_ONE_KERNEL = 1 << 2
@@ -55,6 +55,7 @@ class HydroConfigC(C.Structure):
         ("comm_id", C.c_void_p),
         ("flags", C.c_uint64),
         ("hg_coef", C.c_double),
+        ("dt_floor", C.c_double),
     ]
 
 
@@ -109,6 +110,7 @@ def load_library(path: str = LIB_PATH) -> C.CDLL:
     L.hydro_comm_unique_id.argtypes = [C.c_void_p]
     L.hydro_peer_export.argtypes = [C.c_void_p, C.c_void_p, C.POINTER(C.c_size_t)]
     L.hydro_peer_import.argtypes = [C.c_void_p, C.c_void_p, C.c_size_t]
+    L.hydro_peer_detach.argtypes = [C.c_void_p]
     L.hydro_time_kernels.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_double)]
     L.hydro_kernels_per_cycle.argtypes = [C.c_void_p]
     L.hydro_strerror.restype = C.c_char_p
@@ -160,6 +162,8 @@ class HydroConfig:
                                   # slabs from its own epilogue, HYDRO_FLAG_HALO_FUSED)
     hg_coef: float = 0.0          # viscous hourglass kappa (reading R17); > 0 runs
                                   # the split kernels
+    dt_floor: float = 0.0         # dt-collapse floor (reading R23): > 0 absolute, 0 = 1e-6 dt^0,
+                                  # < 0 none; below it a run halts with EDTMIN
 
 
 class HydroError(RuntimeError):
@@ -190,7 +194,7 @@ def _cfg_struct(cfg: HydroConfig, keep: list, comm_id: Optional[bytes] = None) -
         keep.append(arr)
         c.rank_weight = arr.ctypes.data_as(C.POINTER(C.c_double))
     for k in ("gamma", "q_lin", "q_quad", "cfl", "c_vol", "dt_growth", "dt_max", "dt_init",
-              "t_stop", "dt_first", "t0", "rho0", "e0", "sedov_energy", "hg_coef"):
+              "t_stop", "dt_first", "t0", "rho0", "e0", "sedov_energy", "hg_coef", "dt_floor"):
         setattr(c, k, float(getattr(cfg, k)))
     c.reflect_mask = int(cfg.reflect_mask)
     c.init_kind = {"sedov": 0, "user": 1, "user_mass": 2}[cfg.init]
@@ -451,11 +455,12 @@ class Hydro:
             raise HydroError(rc, "domain_bytes")
         return int(n.value)
 
-    def pack_domain(self, dom: int):
-        """hydro_domain_pack into a new CUDA uint8 tensor (this rank must own ``dom``)."""
+    def pack_domain(self, dom: int, out=None):
+        """hydro_domain_pack into ``out`` (a uint8 tensor on the device or in page-locked host
+        memory) or a new CUDA uint8 tensor (this rank must own ``dom``)."""
         import torch
-        buf = torch.empty(self.domain_bytes(dom), dtype=torch.uint8,
-                          device=f"cuda:{self.cfg.device}")
+        buf = out if out is not None else torch.empty(
+            self.domain_bytes(dom), dtype=torch.uint8, device=f"cuda:{self.cfg.device}")
         rc = self._L.hydro_domain_pack(self._h, int(dom), C.c_void_p(buf.data_ptr()), buf.numel(),
                                        None)
         if rc != 0:
@@ -577,13 +582,24 @@ class Hydro:
         return out, [_info(infos[b]) for b in range(nb)]
 
     def close(self):
+        """Destroy the context (collective).  Peer transport: detach from the other ranks'
+        memory, barrier, then free (hydro_peer_detach; freeing memory another process still
+        maps is undefined in CUDA)."""
         if getattr(self, "_h", None):
+            if self.cfg.nranks > 1 and self.cfg.transport == "peer":
+                import torch.distributed as dist
+                self._L.hydro_peer_detach(self._h)
+                if dist.is_available() and dist.is_initialized():
+                    dist.barrier(group=self._group)
             self._L.hydro_destroy(self._h)
             self._h = None
 
     def __del__(self):
+        # garbage collection is not collective: free without the cross-rank barrier
         try:
-            self.close()
+            if getattr(self, "_h", None):
+                self._L.hydro_destroy(self._h)
+                self._h = None
         except Exception:
             pass
 

@@ -93,9 +93,11 @@ def test_kernels_per_cycle_counts_the_fused_exchange(monkeypatch):
 @pytest.mark.parametrize("mode", ["1", "2", "3"])
 def test_overlapped_halo_copy_bitwise(mode, monkeypatch):
     """Per-source-domain halo copies launched right after each domain's node/energy stage
-    (HYDRO_HALO_OVERLAP=1: on its node-stage stream; 2: on a dedicated halo stream, the
-    default) equal the single copy after the join and the undecomposed run bitwise, with more
-    domains than node-stage streams (uneven cuts, 1-zone-thick domains)."""
+    (HYDRO_HALO_OVERLAP=1: on its node-stage stream; 2: on a dedicated halo stream; 3: one copy
+    per node-stage stream after its last domain, the default when each of the 4 streams holds
+    at most 2 domains, else 0 = one copy after the join) equal the single copy after the join
+    and the undecomposed run bitwise, with more domains than node-stage streams (uneven cuts,
+    1-zone-thick domains)."""
     n = (24, 20, 18)
     cuts = [[0, 5, 13, 24], [0, 1, 20], [0, 9, 10, 18]]
     kw = dict(n=n, ndom=(3, 2, 3), cuts=cuts, init="user", user=jittered_state(n, 9),

@@ -155,18 +155,27 @@ def test_sedov_with_hourglass_conserves_energy():
 
 
 def test_long_sedov_needs_hourglass_control():
-    """Characterisation (DESIGN.md §13 f1): without hourglass control the SG scheme lets a zone
-    next to the blast origin be crushed after ~1000 cycles (dt collapses by many orders while
-    the run is formally healthy); with kappa = 0.03 the same run keeps a normal dt.  Seen
-    identically on the GPU at 448^3 (tools/sedov_front.py).  A regression guard on the scheme's
-    behaviour, not a pin of its values."""
+    """Characterisation (DESIGN.md §13 f1, reading R23): without hourglass control the SG scheme
+    lets a zone next to the blast origin be crushed after ~1000 cycles; dt collapses by many
+    orders while every volume stays positive.  With no floor (dt_floor < 0) the run freezes
+    silently; with the default floor (1e-6 dt^0) it halts with EDTMIN; with kappa = 0.03 the
+    same run keeps a normal dt.  Seen identically on the GPU at 448^3 (tools/sedov_front.py).
+    A regression guard on the scheme's behaviour, not a pin of its values."""
     n, h = 12, 1.2 / 448
     dts = {}
     for kappa in (0.0, 0.03):
-        o = Oracle(OracleConfig(n=(n, n, n), extent=(h * n,) * 3, hg_coef=kappa))
+        o = Oracle(OracleConfig(n=(n, n, n), extent=(h * n,) * 3, hg_coef=kappa, dt_floor=-1.0))
         dt0 = o.step(100)["dt"]
         info = o.step(1200)
         assert info["status"] == 0
         dts[kappa] = info["dt"] / dt0
-    assert dts[0.0] < 1e-6      # collapsed
+    assert dts[0.0] < 1e-6      # collapsed, silently
     assert dts[0.03] > 0.1      # healthy
+    o = Oracle(OracleConfig(n=(n, n, n), extent=(h * n,) * 3))
+    info = o.step(2500)  # the floor is crossed at cycle 1295
+    assert info["status"] == -7 and 100 < info["cycle"] < 2500 and info["bad_zone"] == -1
+    assert info["dt_min_zone"] < 1e-6 * o_dt0(n, h)
+
+
+def o_dt0(n, h):
+    return Oracle(OracleConfig(n=(n, n, n), extent=(h * n,) * 3)).info()["dt"]
