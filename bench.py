@@ -196,6 +196,45 @@ def oracle_baseline(h, budget_s=12.0):
                       f"single-threaded after 1 warm-up cycle ({el:.1f} s)"}
 
 
+def _oracle_worker(h, seconds, q):
+    import oracle
+    from oracle import OracleConfig
+    s = 64
+    o = oracle.Oracle(OracleConfig(n=(s, s, s), extent=(h * s,) * 3))
+    o.step(1)
+    t0, cyc = time.perf_counter(), 0
+    while time.perf_counter() - t0 < seconds:
+        o.step(1)
+        cyc += 1
+    q.put(s ** 3 * cyc / (time.perf_counter() - t0))
+    o.close()
+
+
+def hetero_model(h, gpu_value, seconds=6.0):
+    """SURVEY §8f row f3 (host cores computing thin slabs
+    beside the GPUs, "up to 18 %"), not built; measured instead of modelled: one oracle process
+    per host core runs concurrently (the paper's CPU-only mode, one domain per core), and the
+    aggregate is what the host could add in the ideal case (no halo cost, perfect split)."""
+    import multiprocessing as mp
+    cores = len(os.sched_getaffinity(0))
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_oracle_worker, args=(h, seconds, q)) for _ in range(cores)]
+    for p in ps:
+        p.start()
+    rates = [q.get(timeout=600) for _ in ps]
+    for p in ps:
+        p.join()
+    agg = sum(rates)
+    return {"host_cores": cores, "all_cores_zone_cycles_per_s": agg,
+            "per_core_mean": agg / cores, "gpu_value": gpu_value,
+            "ideal_gain_frac": agg / gpu_value,
+            "note": "row f3 not built: the paper's cooperative mode gains up to 18 percent on "
+                    "K80/P100 nodes; here all host cores running the CPU reference concurrently "
+                    f"(one 64^3 Sedov box per core, {seconds:.0f} s) could add this fraction of "
+                    "the GPU's rate before any host<->device halo cost"}
+
+
 def run_reference(args):
     ws, rank, _ = dist_env()
     if rank != 0:
@@ -568,7 +607,8 @@ def main():
         r2 = Run(args, args.second, ngpu, rank, local, dist, share)
         v2 = r2.timed()
         roof2 = r2.roofline()
-        second = {"workload": r2.desc, "value": v2, "unit": UNIT, "ms_per_step": r2.ms,
+        second = {"workload": r2.desc, "value": v2, "unit": UNIT,
+                  "ms_per_step": r2.ms / args.steps,
                   "steps": args.steps, "warmup": args.warmup, "scaling": r2.scaling,
                   "mesh": list(r2.kw["n"]), "domains": list(r2.cfg.ndom), "zones": r2.zones,
                   "roofline": {k: roof2[k] for k in ("bound", "achieved", "peak", "unit", "frac",
@@ -579,9 +619,11 @@ def main():
 
     check = None if args.no_selfcheck else selfcheck(args, args.config, ngpu, rank, local, dist)
     nccl = nccl_leg(args, args.config, ngpu, rank, local, dist, share)
-    cpu = None
+    cpu = hetero = None
     if rank == 0 and not args.no_cpu_baseline:
         cpu = oracle_baseline(workload(args.config, ngpu)[3])
+        if ngpu == 1:
+            hetero = hetero_model(workload(args.config, ngpu)[3], value)
     if dist:
         dist.barrier()
     if rank == 0:
@@ -592,7 +634,7 @@ def main():
             "dtype": "f64", "data": "synthetic", "config": line_cfg,
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": main_run["clocks"],
             "gpu_launches": main_run["launches"], "kernel_ms": main_run["kt"],
-            "selfcheck": check, "nccl_check": nccl,
+            "selfcheck": check, "nccl_check": nccl, "hetero_host_cpu": hetero,
             args.second or "second": second,
         }
         print(json.dumps(line), flush=True)

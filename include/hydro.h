@@ -77,6 +77,12 @@ enum {
                                              its own epilogue instead of the separate copy / push
                                              kernels after it (correct, measured
                                              slower on B200, so opt-in) */
+#define HYDRO_FLAG_STRICT (1ull << 5)     /* the split pipeline evaluated in the canonical
+                                             operation order of SURVEY §8c (readings R12, R13),
+                                             compiled without FMA contraction: BITWISE equal to
+                                             the oracle (hg_coef = 0; with hg_coef > 0 to within
+                                             the rounding of cbrt).  A checking path, not a
+                                             fast one. */
 
 typedef struct {
   int32_t abi_version;          /* must be HYDRO_ABI_VERSION */

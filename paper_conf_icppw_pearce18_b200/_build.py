@@ -29,10 +29,17 @@ def sources():
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cpp")))
 
 
+def strict_sources():
+    """STRICT path (HYDRO_FLAG_STRICT): compiled on its own without FMA contraction (reading
+    R12), so its operation order is exactly the written one."""
+    return sorted(glob.glob(os.path.join(CSRC, "strict", "*.cu")))
+
+
 def _stale():
     if not os.path.exists(LIB):
         return True
-    deps = sources() + glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh"))
+    deps = (sources() + strict_sources() + glob.glob(os.path.join(CSRC, "*.h")) +
+            glob.glob(os.path.join(CSRC, "*.cuh")))
     deps.append(os.path.join(ROOT, "include", "hydro.h"))
     t = os.path.getmtime(LIB)
     return any(os.path.getmtime(p) > t for p in deps)
@@ -44,10 +51,21 @@ def build(force: bool = False, verbose: bool = False) -> str:
     nccl = _nccl_dir()
     nvcc = os.environ.get("NVCC", "nvcc")
     extra = os.environ.get("HYDRO_NVCC_FLAGS", "").split()
+    objs = []
+    for src in strict_sources():
+        obj = os.path.join(CSRC, "strict", os.path.basename(src)[:-3] + ".o")
+        c = [nvcc, "-c", *extra, "-Xcompiler", "-fPIC", "-O3", "-std=c++17", "-lineinfo", *ARCH,
+             "-fmad=false", "-prec-div=true", "-prec-sqrt=true",
+             "-I", os.path.join(ROOT, "include"), "-o", obj, src]
+        r = subprocess.run(c, capture_output=True, text=True)
+        if r.returncode != 0:
+            sys.stderr.write(r.stdout + r.stderr)
+            raise RuntimeError("nvcc failed (strict)")
+        objs.append(obj)
     cmd = [nvcc, "-shared", *extra, "-Xcompiler", "-fPIC", "-O3", "-std=c++17", "-lineinfo", *ARCH,
            "-Xptxas", "-v" if verbose else "-O3",
            "-I", os.path.join(ROOT, "include"), "-I", os.path.join(nccl, "include"),
-           "-o", LIB + ".tmp", *sources(),
+           "-o", LIB + ".tmp", *sources(), *objs,
            "-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
            "-Xlinker", "-rpath=" + os.path.join(nccl, "lib")]
     r = subprocess.run(cmd, capture_output=True, text=True)

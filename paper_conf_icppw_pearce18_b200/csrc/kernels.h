@@ -87,6 +87,16 @@ void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, cudaStrea
 void launch_node_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 void launch_energy_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 
+// STRICT path (HYDRO_FLAG_STRICT; strict/kernel_strict.cu, compiled with -fmad=false): the
+// split pipeline in the canonical operation order of SURVEY §8c, bitwise equal to the oracle.
+void launch_strict_init_zones(const DomView &d, int kind, double rho0, double e0, double E,
+                              cudaStream_t s);
+void launch_strict_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+void launch_strict_zone(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+void launch_strict_node(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+void launch_strict_energy(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+void launch_strict_derive(const DomView &d, const Phys &ph, cudaStream_t s);
+
 // TMA descriptors of one domain and parity: the six node-state arrays (x,y,z,u,v,w), the
 // constant nodal 8/mass array and the
 // zone arrays m, e, P (box = the kernel's zone tile).

@@ -91,6 +91,7 @@ struct hydro_ctx {
   int graph_k = 1;
   int parity = 0;
   bool split = false;
+  bool strict = false;  // HYDRO_FLAG_STRICT: the split pipeline in the oracle's operation order
   bool one_kernel = false;
   bool use_graph = true;
   int failed = 0;
@@ -479,20 +480,33 @@ int build_push_tables(hydro_ctx *h) {
   return HYDRO_OK;
 }
 
+// Split pipeline (plain or STRICT): zone kernels of every domain, the dt / error reduction,
+// then node and energy kernels.
+int enqueue_split(hydro_ctx *h, int par, cudaStream_t s) {
+  for (LocalDom &D : h->doms) {
+    if (h->strict) launch_strict_zone(D.view[par], h->ph, h->st, s);
+    else launch_zone_split(D.view[par], h->ph, h->st, s);
+  }
+  if (h->comm) {
+    int rc = comm_dt_min(h->comm, h->st, s);
+    if (rc) return set_err(h, rc, "dt allreduce failed");
+  }
+  for (LocalDom &D : h->doms) {
+    if (h->strict) launch_strict_node(D.view[par], h->ph, h->st, s);
+    else launch_node_split(D.view[par], h->ph, h->st, s);
+  }
+  for (LocalDom &D : h->doms) {
+    if (h->strict) launch_strict_energy(D.view[par], h->ph, h->st, s);
+    else launch_energy_split(D.view[par], h->ph, h->st, s);
+  }
+  return HYDRO_OK;
+}
+
 // Enqueue one cycle on stream s reading parity `par`.
 int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
-  for (LocalDom &D : h->doms) {
-    if (h->split) {
-      launch_zone_split(D.view[par], h->ph, h->st, s);
-    }
-  }
   if (h->split) {
-    if (h->comm) {
-      int rc = comm_dt_min(h->comm, h->st, s);
-      if (rc) return set_err(h, rc, "dt allreduce failed");
-    }
-    for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
-    for (LocalDom &D : h->doms) launch_energy_split(D.view[par], h->ph, h->st, s);
+    int rc = enqueue_split(h, par, s);
+    if (rc) return rc;
   } else if (h->one_kernel) {
     for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
     if (h->comm) {
@@ -670,7 +684,8 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
   h->ph.reflect_mask = cfg->reflect_mask;
   h->ph.hg = cfg->hg_coef;
   // hourglass control (f1) needs per-corner forces, which only the split kernels carry
-  h->split = (cfg->flags & HYDRO_FLAG_SPLIT) != 0 || cfg->hg_coef > 0.0;
+  h->strict = (cfg->flags & HYDRO_FLAG_STRICT) != 0;
+  h->split = (cfg->flags & HYDRO_FLAG_SPLIT) != 0 || cfg->hg_coef > 0.0 || h->strict;
   h->one_kernel = !h->split && (cfg->flags & HYDRO_FLAG_ONE_KERNEL) != 0;
   h->use_graph = (cfg->flags & HYDRO_FLAG_NO_GRAPH) == 0;
   h->device = cfg->device;
@@ -898,11 +913,23 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
                                 cfg->init_kind == HYDRO_INIT_USER_MASS);
            if (r) return r;
          }
-         for (LocalDom &D : h->doms)
-           launch_init_zones(D.view[0], cfg->init_kind, cfg->rho0, cfg->e0, cfg->sedov_energy,
-                             h->stream);
+         for (LocalDom &D : h->doms) {
+           if (h->strict)
+             launch_strict_init_zones(D.view[0], cfg->init_kind, cfg->rho0, cfg->e0,
+                                      cfg->sedov_energy, h->stream);
+           else
+             launch_init_zones(D.view[0], cfg->init_kind, cfg->rho0, cfg->e0, cfg->sedov_energy,
+                               h->stream);
+         }
          for (LocalDom &D : h->doms) launch_nodal_mass(D.view[0], h->stream);
-         for (LocalDom &D : h->doms) launch_dt0(D.view[0], h->ph, h->st, h->stream);
+         for (LocalDom &D : h->doms) {
+           if (h->strict) {  // dt^0, then the other parity := this one (node kernel, dt = 0)
+             launch_strict_dt0(D.view[0], h->ph, h->st, h->stream);
+             launch_strict_node(D.view[0], h->ph, h->st, h->stream);
+           } else {
+             launch_dt0(D.view[0], h->ph, h->st, h->stream);
+           }
+         }
          if (h->comm) {
            int r = comm_dt_min(h->comm, h->st, h->stream);
            if (r) return set_err(h, r, "dt allreduce failed");
@@ -1093,7 +1120,10 @@ int hydro_get_box(hydro_ctx *h, const int64_t lo[3], const int64_t hi[3], uint32
   const int par = h->parity;
   const bool derived = (mask & (HYDRO_F_RHO | HYDRO_F_P | HYDRO_F_Q | HYDRO_F_C | HYDRO_F_VOL)) != 0;
   if (derived)
-    for (LocalDom &D : h->doms) launch_derive(D.view[par], h->ph, h->stream);
+    for (LocalDom &D : h->doms) {
+      if (h->strict) launch_strict_derive(D.view[par], h->ph, h->stream);
+      else launch_derive(D.view[par], h->ph, h->stream);
+    }
   const int64_t bn[3] = {hi[0] - lo[0] + 1, hi[1] - lo[1] + 1, hi[2] - lo[2] + 1};
   const int64_t bz[3] = {hi[0] - lo[0], hi[1] - lo[1], hi[2] - lo[2]};
   for (LocalDom &D : h->doms) {
@@ -1396,10 +1426,8 @@ int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
     CK(cudaEventRecord(ev[0], s));
     CK(cudaEventRecord(ev[4], s));
     if (h->split) {
-      for (LocalDom &D : h->doms) launch_zone_split(D.view[par], h->ph, h->st, s);
-      if (h->comm && comm_dt_min(h->comm, h->st, s)) return HYDRO_ENCCL;
-      for (LocalDom &D : h->doms) launch_node_split(D.view[par], h->ph, h->st, s);
-      for (LocalDom &D : h->doms) launch_energy_split(D.view[par], h->ph, h->st, s);
+      int rc = enqueue_split(h, par, s);
+      if (rc) return rc;
     } else if (h->one_kernel) {
       for (LocalDom &D : h->doms) launch_cycle_fused(D.view[par], D.maps[par], h->ph, h->st, fold_finalize(h), s);
       if (h->comm && comm_dt_min(h->comm, h->st, s)) return HYDRO_ENCCL;

@@ -28,6 +28,7 @@ FLAG_SPLIT = 1 << 1
 FLAG_ONE_KERNEL = 1 << 2
 FLAG_PEER = 1 << 3
 FLAG_HALO_FUSED = 1 << 4
+FLAG_STRICT = 1 << 5
 
 STATUS = {0: "ok", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENCCL", -5: "ETANGLED",
           -6: "ENONFINITE", -7: "EDTMIN", -8: "ESTATE"}
@@ -153,7 +154,9 @@ class HydroConfig:
     nranks: int = 1
     device: int = 0
     path: str = "two"             # "two" (zone + node/energy kernels), "one" (one fused kernel),
-                                  # "split" (plain 3-kernel pipeline, HYDRO_FLAG_SPLIT)
+                                  # "split" (plain 3-kernel pipeline, HYDRO_FLAG_SPLIT),
+                                  # "strict" (the split pipeline in the oracle's canonical
+                                  # operation order without FMA: bitwise, HYDRO_FLAG_STRICT)
     graph: bool = True            # CUDA graphs (HYDRO_FLAG_NO_GRAPH when False)
     transport: str = "nccl"       # nranks > 1: "nccl" (NCCL send/recv + allreduce) or "peer"
                                   # (CUDA IPC peer stores + mailbox reduction; ranks may share a GPU)
@@ -211,6 +214,7 @@ def _cfg_struct(cfg: HydroConfig, keep: list, comm_id: Optional[bytes] = None) -
         c.comm_id = C.cast(buf, C.c_void_p)
     c.flags = ((0 if cfg.graph else FLAG_NO_GRAPH) | (FLAG_SPLIT if cfg.path == "split" else 0)
                | (FLAG_ONE_KERNEL if cfg.path == "one" else 0)
+               | (FLAG_STRICT if cfg.path == "strict" else 0)
                | (FLAG_PEER if cfg.transport == "peer" else 0)
                | (FLAG_HALO_FUSED if cfg.halo == "fused" else 0))
     return c
