@@ -692,6 +692,12 @@ __global__ void __launch_bounds__(CTile<TX, TY>::NTHR, 1)
 // (measured: 128^3 85.3 vs 89.7 us with TY = 11, weak 384^3 slabs 499.7 vs 473.8 with TY = 12).
 // The grouped launch and the one-kernel variant use CTY.
 constexpr int CTX = 32, CTY = 12, CTY_ALT = 11;
+// one-kernel variant's tile height (HYDRO_FUSED_TY at build time; default CTY): smaller tiles
+// give each thread more registers (NTHR threads at one CTA per SM)
+#ifndef HYDRO_FUSED_TY
+#define HYDRO_FUSED_TY 12
+#endif
+constexpr int FTY = HYDRO_FUSED_TY;
 
 // z-chunk length of the chunked schedule: minimise (waves of CTAs) x (planes per CTA incl. the
 // 2 warm-up planes + a fixed per-chunk overhead of 1.4 plane-equivalents: pipeline fill and
@@ -786,12 +792,12 @@ void launch(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st
 
 }  // namespace
 
-size_t fused_smem_bytes() { return CTile<CTX, CTY>::BYTES; }
-int fused_box_y() { return CTile<CTX, CTY>::BYN; }
-int node_box_y(int ty) { return ty == CTY_ALT ? CTile<CTX, CTY_ALT>::BYN : CTile<CTX, CTY>::BYN; }
+size_t fused_smem_bytes() { return CTile<CTX, FTY>::BYTES; }
+int fused_box_y() { return CTile<CTX, FTY>::BYN; }
+int node_box_y(int ty) { return ty + 3; }  // CTile<CTX, ty>::BYN
 int cycle_zone_box_x() { return CTile<CTX, CTY>::ZBX; }
 int cycle_zone_box_y(int ty) {
-  return ty == CTY_ALT ? CTile<CTX, CTY_ALT>::ZBY : CTile<CTX, CTY>::ZBY;
+  return ty + 2;  // CTile<CTX, ty>::ZBY
 }
 
 int node_tile_ty(int n0, int n1, int n2) {
@@ -804,8 +810,9 @@ int node_tile_ty(int n0, int n1, int n2) {
 
 void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                         int fold_finalize, cudaStream_t s) {
-  launch<true, CTY>(d, maps, ph, st, fold_finalize, nullptr, 0, s);
+  launch<true, FTY>(d, maps, ph, st, fold_finalize, nullptr, 0, s);
 }
+int fused_tile_ty() { return FTY; }
 
 void launch_node_energy(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
                         int fold_finalize, const PushSlab *push, int npush, int ty,

@@ -343,13 +343,14 @@ __global__ void __launch_bounds__(ZBX *ZBY, HYDRO_ZONE_MINB)
 }
 
 
-// Tiling of one domain's zone stage: ghost ring only on sides with a neighbouring domain.
-ZoneTask zone_task(const DomView &d, int slot) {
+// Tiling of one domain's zone stage: ghost ring only on sides with a neighbouring domain whose
+// ring bit is set (ring zones owned by a domain of this GPU get their P by a copy instead).
+ZoneTask zone_task(const DomView &d, int slot, uint8_t ring) {
   ZoneTask T = {};
   T.slot = slot;
   for (int a = 0; a < 3; ++a) {
-    T.zlo[a] = d.lo[a] > 0 ? -1 : 0;
-    T.zhi[a] = d.lo[a] + d.n[a] < d.N[a] ? d.n[a] + 1 : d.n[a];
+    T.zlo[a] = (d.lo[a] > 0 && (ring >> (2 * a) & 1u)) ? -1 : 0;
+    T.zhi[a] = (d.lo[a] + d.n[a] < d.N[a] && (ring >> (2 * a + 1) & 1u)) ? d.n[a] + 1 : d.n[a];
   }
   T.tcols = (T.zhi[0] - T.zlo[0] + ZBX - 1) / ZBX;
   const int ty = (T.zhi[1] - T.zlo[1] + ZBY - 1) / ZBY;
@@ -382,10 +383,10 @@ int zone_slots() {  // per device: the shared-memory opt-in is a per-device attr
 
 int zone_box_y() { return ZNY; }
 
-void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                       cudaStream_t s) {
+void launch_zone_stage(const DomView &d, const NodeMaps &maps, uint8_t ring, const Phys &ph,
+                       DevState *st, cudaStream_t s) {
   const int slots = zone_slots();
-  ZoneTask T = zone_task(d, 0);
+  ZoneTask T = zone_task(d, 0, ring);
   // Default: the persistent linearised split (measured 67 vs 70 us for the best chunking at
   // 128^3).  HYDRO_KZ_ZONE=k: the chunked schedule with k planes per CTA (A/B measurement).
   static const int kz_env = getenv("HYDRO_KZ_ZONE") ? atoi(getenv("HYDRO_KZ_ZONE")) : 0;
@@ -403,10 +404,11 @@ void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, D
              T.units, kz, ph, st);
 }
 
-void zone_group_tasks(const DomView *views_host, int n, ZoneTask *out, int64_t *Wtot) {
+void zone_group_tasks(const DomView *views_host, const uint8_t *rings, int n, ZoneTask *out,
+                      int64_t *Wtot) {
   int64_t u = 0;
   for (int i = 0; i < n; ++i) {
-    out[i] = zone_task(views_host[i], i);
+    out[i] = zone_task(views_host[i], i, rings[i]);
     out[i].u0 = u;
     u += out[i].units;
   }

@@ -35,7 +35,8 @@ cudaError_t launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, 
 struct HaloCopy {  // one chunk of an intra-GPU ghost slab copy (global boxes, half-open)
   int32_t dst, src;  // local domain slots
   int64_t nlo[3], nhi[3], zlo[3], zhi[3];
-  int32_t kind;         // 0: the node slab (x,y,z,u,v,w), 1: the zone slab (e)
+  int32_t kind;         // 0: the node slab (x,y,z,u,v,w), 1: the zone slab (e), 2: the zone
+                        // slab of the current cycle's P (ring zones the zone stage skips)
   int32_t start, count; // elements [start, start+count) of that slab, x fastest
 };
 constexpr int HALO_CHUNK = 2048;  // elements per chunk (one CTA of 256 threads)
@@ -112,6 +113,7 @@ void launch_cycle_fused(const DomView &d, const NodeMaps &maps, const Phys &ph, 
                         int fold_finalize, cudaStream_t s);
 size_t fused_smem_bytes();
 int fused_box_y();
+int fused_tile_ty();  // tile height of the one-kernel variant
 
 // Two-kernel cycle (default path): zone stage (P, dt) then node/energy stage.
 // Node/energy-stage work of one domain in a grouped launch (kernel_cycle.cu): x-tiles, columns,
@@ -129,12 +131,16 @@ void launch_node_energy_group(const NodeTask *tasks_dev, int ntasks, int nctas,
 // Grouped zone stage over all local domains (one persistent launch): tasks from
 // zone_group_tasks (host), copied to the device by the caller; views_dev / maps_dev indexed by
 // ZoneTask::slot.
-void zone_group_tasks(const DomView *views_host, int n, ZoneTask *out, int64_t *Wtot);
+// rings[i]: bit 2a+h = compute the ghost-zone ring of domain i on side h (0 low, 1 high) of
+// axis a (where a neighbour exists); clear = its P comes from the owning local domain by a
+// kind-2 halo copy after the zone stage (runtime.cu)
+void zone_group_tasks(const DomView *views_host, const uint8_t *rings, int n, ZoneTask *out,
+                      int64_t *Wtot);
 void launch_zone_stage_group(const DomView *views_dev, const NodeMaps *maps_dev,
                              const ZoneTask *tasks_dev, int64_t Wtot, const Phys &ph,
                              DevState *st, cudaStream_t s);
-void launch_zone_stage(const DomView &d, const NodeMaps &maps, const Phys &ph, DevState *st,
-                       cudaStream_t s);
+void launch_zone_stage(const DomView &d, const NodeMaps &maps, uint8_t ring, const Phys &ph,
+                       DevState *st, cudaStream_t s);
 // push/npush: this domain's fused-halo slabs (nullptr/0: none; the caller then exchanges the
 // ghost layer with launch_halo_copy / the transports).
 // ty: node-stage tile height (node_tile_ty; the TMA maps must be built with its boxes).

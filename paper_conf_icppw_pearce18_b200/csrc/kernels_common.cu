@@ -314,9 +314,13 @@ __global__ void k_halo_copy(const DomView *views, const HaloCopy *chunks) {
                                (int)(p.zlo[2] - D.lo[2]));
     const int zs0 = (int)S.zid((int)(p.zlo[0] - S.lo[0]), (int)(p.zlo[1] - S.lo[1]),
                                (int)(p.zlo[2] - S.lo[2]));
+    // kind 1: next-parity e; kind 2: this cycle's P (zone-stage ring zones, before the node
+    // stage)
+    const double *src = p.kind == 2 ? S.P : S.en;
+    double *dst = p.kind == 2 ? D.P : D.en;
     for (int t = p.start + threadIdx.x; t < p.start + p.count; t += blockDim.x) {
       const int a = t % zx, r = t / zx, b = r % zy, c = r / zy;
-      D.en[zd0 + c * zdsxy + b * zdsx + a] = __ldg(S.en + zs0 + c * zssxy + b * zssx + a);
+      dst[zd0 + c * zdsxy + b * zdsx + a] = __ldg(src + zs0 + c * zssxy + b * zssx + a);
     }
   }
 }

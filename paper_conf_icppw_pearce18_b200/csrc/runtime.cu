@@ -60,6 +60,11 @@ struct hydro_ctx {
   std::vector<NodeTask> ntasks_host;
   int nctas = 0;
   int n_local_pairs = 0;
+  // zone-stage ghost rings: ring[slot] bit 2a+h = compute the ring on that side;
+  // ring zones owned by another domain of this rank get their P by a copy after the zone stage
+  std::vector<uint8_t> ring;
+  HaloCopy *pcopy_dev = nullptr;
+  int n_pcopy = 0;
   // halo copy overlapped with the other domains' node stages: chunks sorted by source slot, each
   // domain's outgoing slabs copied on its own stream right after its node/energy stage
   // (HYDRO_HALO_OVERLAP=0 for the single copy after the join, A/B)
@@ -187,8 +192,9 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
   const int64_t n0 = D.box.n[0], n1 = D.box.n[1], n2 = D.box.n[2];
   // node-stage tile height: chosen per domain, except for the grouped node launch and the
   // one-kernel variant, which are compiled for the default height only
-  const bool fixed_ty = h->one_kernel || (h->doms.size() > 1 && group_node());
-  D.node_ty = fixed_ty ? 12 : node_tile_ty((int)n0, (int)n1, (int)n2);
+  const bool fixed_ty = h->doms.size() > 1 && group_node();
+  D.node_ty = h->one_kernel ? fused_tile_ty()
+                            : (fixed_ty ? 12 : node_tile_ty((int)n0, (int)n1, (int)n2));
   const int64_t nsx = (n0 + 3 + 3) / 4 * 4, nsxy = nsx * (n1 + 3), nnode = nsxy * (n2 + 3);
   const int64_t zsx = (n0 + 2 + 3) / 4 * 4, zsxy = zsx * (n1 + 2);
   if (nnode >= (int64_t(1) << 31))  // the cycle kernels index a domain's storage with int32
@@ -213,8 +219,6 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
                             D.view[par].u, D.view[par].v, D.view[par].w, D.view[par].mn8};
     const double *zarr[4] = {D.view[par].m, D.view[par].e, D.view[par].P, D.view[par].mi};
     for (int kind = 0; kind < 2; ++kind) {
-      if (kind == 0 && D.node_ty == 12 && fused_box_y() != node_box_y(12))
-        return set_err(h, HYDRO_EINVAL, "fused and node kernels must share a TMA box");
       NodeMaps &M = kind ? D.zmaps[par] : D.maps[par];
       for (int f = 0; f < 11; ++f) {
         const bool zf = f >= 6 && f < 10;
@@ -360,7 +364,11 @@ void launch_zone_stages(hydro_ctx *h, int par, cudaStream_t s) {
     launch_zone_stage_group(h->views_dev[par], h->zmaps_dev[par], h->ztasks_dev, h->zunits,
                             h->ph, h->st, s);
   else
-    for (LocalDom &D : h->doms) launch_zone_stage(D.view[par], D.zmaps[par], h->ph, h->st, s);
+    for (size_t i = 0; i < h->doms.size(); ++i)
+      launch_zone_stage(h->doms[i].view[par], h->doms[i].zmaps[par], h->ring[i], h->ph, h->st,
+                        s);
+  // P of the ring zones the zone stages skipped, from their owners on this GPU
+  if (h->n_pcopy) launch_halo_copy(h->views_dev[par], h->pcopy_dev, h->n_pcopy, s);
 }
 
 // The grouped node/energy launch is measured slower on large domains (512^3 in 8 domains: 695
@@ -749,6 +757,26 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
              CK(cudaMemcpyAsync(h->views_dev[par], vv.data(), sizeof(DomView) * vv.size(),
                                 cudaMemcpyHostToDevice, h->stream));
          }
+         // zone-stage rings: only on sides where a ghost zone is owned by another rank (the
+         // rest is copied from the local owner after the zone stage; HYDRO_PRING=0: always
+         // compute the ring, A/B)
+         {
+           const char *pr = getenv("HYDRO_PRING");
+           const bool skip = !(pr && atoi(pr) == 0) && !h->split && !h->one_kernel;
+           h->ring.assign(h->doms.size(), skip ? 0 : 0x3f);
+           for (const HaloPair &P : h->L.pairs) {
+             const int32_t ds = h->slot_of_dom[P.dst];
+             if (!skip || ds < 0 || h->slot_of_dom[P.src] >= 0) continue;
+             const DomainBox &b = h->doms[ds].box;
+             bool empty = false;
+             for (int a = 0; a < 3; ++a) empty |= P.zhi[a] <= P.zlo[a];
+             if (empty) continue;
+             for (int a = 0; a < 3; ++a) {
+               if (P.zhi[a] <= b.lo[a]) h->ring[ds] |= (uint8_t)(1u << (2 * a));
+               if (P.zlo[a] >= b.lo[a] + b.n[a]) h->ring[ds] |= (uint8_t)(1u << (2 * a + 1));
+             }
+           }
+         }
          // several domains on this GPU: one grouped zone-stage launch covers them all
          // (HYDRO_NO_GROUP=1: one launch per domain, for A/B)
          h->group = h->doms.size() > 1 && !h->split && !h->one_kernel &&
@@ -757,7 +785,7 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
            std::vector<DomView> vv;
            for (LocalDom &D : h->doms) vv.push_back(D.view[0]);
            std::vector<ZoneTask> tasks(vv.size());
-           zone_group_tasks(vv.data(), (int)vv.size(), tasks.data(), &h->zunits);
+           zone_group_tasks(vv.data(), h->ring.data(), (int)vv.size(), tasks.data(), &h->zunits);
            CK(cudaMalloc(&h->ztasks_dev, sizeof(ZoneTask) * tasks.size()));
            CK(cudaMemcpy(h->ztasks_dev, tasks.data(), sizeof(ZoneTask) * tasks.size(),
                          cudaMemcpyHostToDevice));
@@ -781,7 +809,7 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
            CK(cudaMemcpy(h->ntasks_dev, nt.data(), sizeof(NodeTask) * nt.size(),
                          cudaMemcpyHostToDevice));
          }
-         std::vector<HaloCopy> lp;
+         std::vector<HaloCopy> lp, pc;
          std::vector<HaloPair> remote;
          for (const HaloPair &P : h->L.pairs) {
            const bool dst_local = h->slot_of_dom[P.dst] >= 0;
@@ -806,14 +834,16 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
                nn *= P.nhi[a] - P.nlo[a];
                nz *= P.zhi[a] - P.zlo[a];
              }
-             // chunks of HALO_CHUNK elements: the node slab, then the zone slab
-             for (int kind = 0; kind < 2; ++kind) {
+             // chunks of HALO_CHUNK elements: the node slab, then the zone slab; the zone slab
+             // once more for P when the destination's zone stage skips its ring there
+             for (int kind = 0; kind < 3; ++kind) {
+               if (kind == 2 && h->ring[c.dst] == 0x3f) continue;
                const int64_t total = kind ? nz : nn;
                for (int64_t st = 0; st < total; st += HALO_CHUNK) {
                  c.kind = kind;
                  c.start = (int32_t)st;
                  c.count = (int32_t)std::min<int64_t>(HALO_CHUNK, total - st);
-                 lp.push_back(c);
+                 (kind == 2 ? pc : lp).push_back(c);
                }
              }
            } else if (dst_local || src_local) {
@@ -885,6 +915,12 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
          if (h->fused_halo) {
            int r = build_push_tables(h);
            if (r) return r;
+         }
+         if (!pc.empty()) {
+           CK(cudaMalloc(&h->pcopy_dev, sizeof(HaloCopy) * pc.size()));
+           CK(cudaMemcpyAsync(h->pcopy_dev, pc.data(), sizeof(HaloCopy) * pc.size(),
+                              cudaMemcpyHostToDevice, h->stream));
+           h->n_pcopy = (int)pc.size();
          }
          if (!lp.empty()) {
            CK(cudaMalloc(&h->local_pairs_dev, sizeof(HaloCopy) * lp.size()));
@@ -1405,6 +1441,7 @@ int hydro_kernels_per_cycle(const hydro_ctx *h) {
   } else if (h->n_local_pairs > 0 && !h->fused_halo) {
     k += 1;  // intra-GPU halo copy
   }
+  if (h->n_pcopy) k += 1;           // P of skipped zone-stage rings
   if (!fold_finalize(h)) k += 1;     // finalize
   if (h->comm) k += comm_kernels_per_cycle(h->comm);
   if (h->peer) k += peer_kernels_per_cycle(h->peer, !h->fused_halo);
@@ -1490,6 +1527,7 @@ int hydro_destroy(hydro_ctx *h) {
   if (!h) return HYDRO_OK;
   cudaSetDevice(h->device);
   if (h->stream) cudaStreamSynchronize(h->stream);
+  if (h->pcopy_dev) cudaFree(h->pcopy_dev);
   for (int p = 0; p < 2; ++p) {
     if (h->graph[p]) cudaGraphExecDestroy(h->graph[p]);
     if (h->graphk[p]) cudaGraphExecDestroy(h->graphk[p]);
