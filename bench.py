@@ -522,8 +522,20 @@ def nccl_leg(args, name, ngpu, rank, local, dist, share):
         return {"ran": False, "why": "ranks share one GPU (HYDRO_SHARE_GPU): NCCL refuses"}
     import torch
     from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig, dom_to_rank
+    # a stalled NCCL leg ends in HYDRO_ENCCL after this long (comm_wait polls
+    # ncclCommGetAsyncError), not in a hung bench
+    os.environ.setdefault("HYDRO_NCCL_TIMEOUT_S", "120")
     kw, _, _, _ = workload(name, ngpu)
     packs, ms = {}, {}
+    try:
+        return _nccl_leg_run(args, kw, ngpu, rank, local, dist, torch, Hydro, HydroConfig,
+                             dom_to_rank, packs, ms)
+    except Exception as exc:  # reported in the line, the timed numbers above stand
+        return {"ran": True, "error": f"{type(exc).__name__}: {exc}"[:300]}
+
+
+def _nccl_leg_run(args, kw, ngpu, rank, local, dist, torch, Hydro, HydroConfig, dom_to_rank,
+                  packs, ms):
     for tr in ("peer", "nccl"):
         cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, path=args.path, transport=tr,
                           hg_coef=args.hg, halo=args.halo, **kw)

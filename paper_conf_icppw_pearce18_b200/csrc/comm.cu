@@ -2,6 +2,7 @@
 #include <nccl.h>
 
 #include <chrono>
+#include <cstdlib>
 #include <cstring>
 #include <thread>
 
@@ -74,6 +75,10 @@ struct Comm {
   int64_t send_total = 0, recv_total = 0;
   DomView *views_dev[2] = {nullptr, nullptr};
   unsigned long long *red_dev = nullptr;  // [4]: the S9 allreduce words
+  // overlapped dt reduction (HYDRO_DT_OVERLAP, default on): own communicator and stream
+  ncclComm_t dtcomm = nullptr;
+  cudaStream_t cs = nullptr;
+  cudaEvent_t fork = nullptr, join = nullptr;
 };
 
 int comm_unique_id(void *out128) {
@@ -130,6 +135,20 @@ int comm_create(Comm **out, const hydro_config *cfg, const Layout &L,
     if (e != cudaSuccess) *err = cudaGetErrorString(e);
     return e == cudaSuccess;
   };
+  {
+    const char *ov = getenv("HYDRO_DT_OVERLAP");
+    if (!(ov && atoi(ov) == 0)) {
+      if (ncclCommSplit(c->nccl, 0, cfg->rank, &c->dtcomm, nullptr) != ncclSuccess) {
+        *err = "ncclCommSplit failed";
+        return HYDRO_ENCCL;
+      }
+      int lo = 0, hi = 0;
+      cudaDeviceGetStreamPriorityRange(&lo, &hi);
+      if (!ck(cudaStreamCreateWithPriority(&c->cs, cudaStreamNonBlocking, hi))) return HYDRO_ECUDA;
+      if (!ck(cudaEventCreateWithFlags(&c->fork, cudaEventDisableTiming))) return HYDRO_ECUDA;
+      if (!ck(cudaEventCreateWithFlags(&c->join, cudaEventDisableTiming))) return HYDRO_ECUDA;
+    }
+  }
   if (!ck(cudaMalloc(&c->red_dev, 4 * sizeof(unsigned long long)))) return HYDRO_ECUDA;
   if (c->send_total) {
     if (!ck(cudaMalloc(&c->sendbuf, c->send_total * sizeof(double)))) return HYDRO_ENOMEM;
@@ -174,6 +193,26 @@ int comm_dt_min(Comm *c, DevState *st, cudaStream_t s) {
   return cudaGetLastError() == cudaSuccess ? HYDRO_OK : HYDRO_ECUDA;
 }
 
+bool comm_dt_overlap(const Comm *c) { return c && c->dtcomm; }
+
+int comm_dt_min_async(Comm *c, DevState *st, cudaStream_t s) {
+  if (!c->dtcomm) return comm_dt_min(c, st, s);
+  if (cudaEventRecord(c->fork, s) != cudaSuccess) return HYDRO_ECUDA;
+  if (cudaStreamWaitEvent(c->cs, c->fork, 0) != cudaSuccess) return HYDRO_ECUDA;
+  k_red_pack<<<1, 1, 0, c->cs>>>(st, c->red_dev);
+  if (ncclAllReduce(c->red_dev, c->red_dev, 4, ncclUint64, ncclMax, c->dtcomm, c->cs) !=
+      ncclSuccess)
+    return HYDRO_ENCCL;
+  k_red_unpack<<<1, 1, 0, c->cs>>>(st, c->red_dev);
+  if (cudaEventRecord(c->join, c->cs) != cudaSuccess) return HYDRO_ECUDA;
+  return cudaGetLastError() == cudaSuccess ? HYDRO_OK : HYDRO_ECUDA;
+}
+
+int comm_dt_join(Comm *c, cudaStream_t s) {
+  if (!c->dtcomm) return HYDRO_OK;
+  return cudaStreamWaitEvent(s, c->join, 0) == cudaSuccess ? HYDRO_OK : HYDRO_ECUDA;
+}
+
 int comm_halo(Comm *c, int par, cudaStream_t s) {
   if (!c->sends.empty())
     k_pack<<<dim3(8, (unsigned)c->sends.size()), 256, 0, s>>>(c->views_dev[par], c->sends_dev,
@@ -204,19 +243,26 @@ int comm_wait(Comm *c, cudaStream_t s, double timeout_s, std::string *err) {
       *err = std::string("stream: ") + cudaGetErrorString(q);
       return HYDRO_ECUDA;
     }
-    ncclResult_t ae = ncclSuccess;
-    if (ncclCommGetAsyncError(c->nccl, &ae) != ncclSuccess || ae != ncclSuccess) {
+    ncclResult_t ae = ncclSuccess, ae2 = ncclSuccess;
+    if (c->dtcomm && (ncclCommGetAsyncError(c->dtcomm, &ae2) != ncclSuccess || ae2 != ncclSuccess))
+      ae = ae2 != ncclSuccess ? ae2 : ncclInternalError;
+    if (ae != ncclSuccess || ncclCommGetAsyncError(c->nccl, &ae) != ncclSuccess ||
+        ae != ncclSuccess) {
       *err = std::string("NCCL asynchronous error: ") + ncclGetErrorString(ae);
+      if (c->dtcomm) ncclCommAbort(c->dtcomm);
       ncclCommAbort(c->nccl);
       c->nccl = nullptr;
+      c->dtcomm = nullptr;
       return HYDRO_ENCCL;
     }
     const double el =
         std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
     if (timeout_s > 0.0 && el > timeout_s) {
       *err = "NCCL wait timed out (a peer rank stalled or died)";
+      if (c->dtcomm) ncclCommAbort(c->dtcomm);
       ncclCommAbort(c->nccl);
       c->nccl = nullptr;
+      c->dtcomm = nullptr;
       return HYDRO_ENCCL;
     }
     if (spin > 64) std::this_thread::sleep_for(std::chrono::microseconds(50));
@@ -229,7 +275,11 @@ int comm_kernels_per_cycle(const Comm *c) {
 
 void comm_destroy(Comm *c) {
   if (!c) return;
+  if (c->dtcomm) ncclCommDestroy(c->dtcomm);
   if (c->nccl) ncclCommDestroy(c->nccl);
+  if (c->cs) cudaStreamDestroy(c->cs);
+  if (c->fork) cudaEventDestroy(c->fork);
+  if (c->join) cudaEventDestroy(c->join);
   cudaFree(c->sendbuf);
   cudaFree(c->recvbuf);
   cudaFree(c->sends_dev);

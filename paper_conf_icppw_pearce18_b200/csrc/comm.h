@@ -29,6 +29,12 @@ int comm_bind_views(Comm *c, const DomView *const *views0, const DomView *const 
                     std::string *err);
 // Global S9 inputs: st->dtz_acc <- min over ranks, st->err <- OR over ranks (in place, on s).
 int comm_dt_min(Comm *c, DevState *st, cudaStream_t s);
+// The same reduction off the critical path (two-kernel path): forked from s after the zone
+// stage onto the communicator's own stream and a second communicator (ncclCommSplit), so it
+// overlaps the node stages (dt_{n+1} is first read by S9); comm_dt_join makes s wait for it.
+int comm_dt_min_async(Comm *c, DevState *st, cudaStream_t s);
+int comm_dt_join(Comm *c, cudaStream_t s);
+bool comm_dt_overlap(const Comm *c);
 // Exchange the next-parity ghost slabs of parity-`par` views with remote neighbours.
 int comm_halo(Comm *c, int par, cudaStream_t s);
 // Wait for stream s while polling the communicator: returns HYDRO_OK once s is

@@ -238,10 +238,20 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
         box[2] = 1;
         cuuint32_t es[3] = {1, 1, 1};
         CUtensorMap *dst = zf ? &M.z[f - 6] : &M.m[f == 10 ? 6 : f];
+        // L2 promotion: the node-stage maps keep 256 B (adjacent CTAs at the same z read the
+        // neighbouring bytes of a promoted line); the persistent zone stage's CTAs sit at
+        // different z, so a promoted line's other half is never reused and its 36-double rows
+        // (288 B) would fetch 512 B (HYDRO_ZPROMO / HYDRO_NPROMO: 0 none, 1 64 B, 2 128 B, 3 256 B)
+        static const int zpromo = getenv("HYDRO_ZPROMO") ? atoi(getenv("HYDRO_ZPROMO")) : 3;
+        static const int npromo = getenv("HYDRO_NPROMO") ? atoi(getenv("HYDRO_NPROMO")) : 3;
+        const CUtensorMapL2promotion promos[4] = {
+            CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_64B,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B};
+        const int pi = std::max(0, std::min(3, (kind && !zf) ? zpromo : npromo));
         CUresult r = encode(dst, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3,
                             const_cast<double *>(zf ? zarr[f - 6] : arr[f == 10 ? 6 : f]), dims, strides, box,
                             es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                            promos[pi], CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
         if (r != CUDA_SUCCESS) return set_err(h, HYDRO_ECUDA, "cuTensorMapEncodeTiled failed");
       }
     }
@@ -523,8 +533,8 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
     }
   } else {
     launch_zone_stages(h, par, s);
-    if (h->comm) {
-      int rc = comm_dt_min(h->comm, h->st, s);
+    if (h->comm) {  // dt_{n+1} is first read by S9: the reduction overlaps the node stages
+      int rc = comm_dt_min_async(h->comm, h->st, s);
       if (rc) return set_err(h, rc, "dt allreduce failed");
     }
     launch_node_stages(h, par, s, h->halo_overlap);
@@ -538,6 +548,10 @@ int enqueue_cycle(hydro_ctx *h, int par, cudaStream_t s) {
   if (h->peer) {  // halo push into the peers (unless fused) + dt / error reduction
     int rc = peer_exchange(h->peer, h->views_dev[par], par, !h->fused_halo, h->st, s);
     if (rc) return set_err(h, rc, "peer exchange failed");
+  }
+  if (h->comm && !h->split && !h->one_kernel) {
+    int rc = comm_dt_join(h->comm, s);
+    if (rc) return set_err(h, rc, "dt allreduce join failed");
   }
   if (!fold_finalize(h)) launch_finalize(h->st, h->ph, s);
   CK(cudaGetLastError());
