@@ -239,10 +239,11 @@ int alloc_domain(hydro_ctx *h, LocalDom &D, bool split) {
         cuuint32_t es[3] = {1, 1, 1};
         CUtensorMap *dst = zf ? &M.z[f - 6] : &M.m[f == 10 ? 6 : f];
         // L2 promotion: the node-stage maps keep 256 B (adjacent CTAs at the same z read the
-        // neighbouring bytes of a promoted line); the persistent zone stage's CTAs sit at
-        // different z, so a promoted line's other half is never reused and its 36-double rows
-        // (288 B) would fetch 512 B (HYDRO_ZPROMO / HYDRO_NPROMO: 0 none, 1 64 B, 2 128 B, 3 256 B)
-        static const int zpromo = getenv("HYDRO_ZPROMO") ? atoi(getenv("HYDRO_ZPROMO")) : 3;
+        // neighbouring bytes of a promoted line; 128/64/none measured 1-2 % slower); the
+        // persistent zone stage's CTAs sit at different z, so a promoted line's other half is
+        // rarely reused: 64 B cuts its DRAM reads at 512^3 from 121 to 94 B/zone (ncu) and its
+        // time by 1 % (HYDRO_ZPROMO / HYDRO_NPROMO: 0 none, 1 64 B, 2 128 B, 3 256 B)
+        static const int zpromo = getenv("HYDRO_ZPROMO") ? atoi(getenv("HYDRO_ZPROMO")) : 1;
         static const int npromo = getenv("HYDRO_NPROMO") ? atoi(getenv("HYDRO_NPROMO")) : 3;
         const CUtensorMapL2promotion promos[4] = {
             CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_64B,

@@ -1,14 +1,18 @@
 """Summarise an ncu --set full report into per-kernel counters used by bench.py's roofline:
 DRAM bytes and executed fp64 (DADD/DMUL/DFMA) thread instructions per launch, per owned zone.
 
-    python tools/ncu_summary.py report.ncu-rep ZONES > profiles/kernel_counters.json
+    python tools/ncu_summary.py report.ncu-rep ZONES [KERNEL=ZONES ...] > profiles/kernel_counters.json
+
+ZONES: owned zones one launch covers; KERNEL=ZONES overrides it per kernel key (e.g. the grouped
+zone stage covers every domain of the GPU, a node-stage launch one domain).
 """
 import csv
 import json
 import subprocess
 import sys
 
-rep, zones = sys.argv[1], float(sys.argv[2])
+rep, zones_all = sys.argv[1], float(sys.argv[2])
+zones_of = {kv.split("=")[0]: float(kv.split("=")[1]) for kv in sys.argv[3:]}
 raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
                      text=True).stdout.splitlines()
 rows = list(csv.reader(raw))
@@ -22,6 +26,7 @@ for vals in rows[2:]:
             "k_node_energy" if "k_cycle<" in name else name.split("(")[0]))
     if key in out:
         continue
+    zones = zones_of.get(key, zones_all)
     def f(k):
         try:
             return float(d[k].replace(",", ""))
@@ -41,6 +46,7 @@ for vals in rows[2:]:
         "duration_us": f("gpu__time_duration.sum") * {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0,
                                                       "us": 1.0, "msecond": 1e3, "ms": 1e3}[units["gpu__time_duration.sum"]],
         "dram_bytes": (rd + wr) * unit, "dram_read_bytes": rd * unit, "dram_write_bytes": wr * unit,
+        "zones_per_launch": zones,
         "dram_bytes_per_zone": (rd + wr) * unit / zones,
         "fp64_inst": fp64, "fp64_inst_per_zone": fp64 / zones,
         "fp64_pipe_pct": f("sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active"),
@@ -53,5 +59,5 @@ for vals in rows[2:]:
         "smem_wavefronts_pct": f("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum"
                                  ".pct_of_peak_sustained_elapsed"),
     }
-json.dump({"report": rep, "zones": zones, "kernels": out}, sys.stdout, indent=1)
+json.dump({"report": rep, "zones": zones_all, "kernels": out}, sys.stdout, indent=1)
 print()

@@ -1,12 +1,15 @@
 """Small runs of every cycle path for compute-sanitizer (memcheck / racecheck / synccheck)."""
 import os
 import sys
-from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig
-from paper_conf_icppw_pearce18_b200.inputs import jittered_state
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig  # noqa: E402
+from paper_conf_icppw_pearce18_b200.inputs import jittered_state  # noqa: E402
 
 n = (40, 30, 20)
 cuts = [[0, 17, 40], [0, 12, 30], [0, 20]]
-for path in sys.argv[1:] or ["two", "one", "split", "hg", "single", "fused", "ty11", "ty12"]:
+for path in sys.argv[1:] or ["two", "one", "split", "strict", "hg", "single", "fused", "ty11",
+                             "ty12"]:
     kw = dict(n=n, ndom=(2, 2, 1), cuts=cuts, init="user", user=jittered_state(n, 3), path=path,
               graph=False)
     if path == "hg":  # hourglass control (split kernels)
