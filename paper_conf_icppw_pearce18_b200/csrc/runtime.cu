@@ -4,6 +4,7 @@
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>  // header-only; ranges show up in nsys / ncu --nvtx
 
 #include <algorithm>
 #include <cmath>
@@ -130,6 +131,12 @@ int set_err(hydro_ctx *h, int code, const std::string &msg) {
   } while (0)
 
 size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+// NVTX range for the duration of a C-ABI call (tracing)
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 }  // namespace
 
@@ -670,6 +677,7 @@ const char *hydro_last_error(const hydro_ctx *h) { return h ? h->err.c_str() : g
 int hydro_comm_unique_id(void *out128) { return comm_unique_id(out128); }
 
 int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
+  NvtxRange nvtx_("hydro_create");
   hydro_ctx *h = nullptr;
   if (!cfg || !out) return set_err(nullptr, HYDRO_EINVAL, "NULL argument");
   *out = nullptr;
@@ -1039,6 +1047,7 @@ int hydro_peer_import(hydro_ctx *h, const void *all, size_t len_per_rank) {
 }
 
 int hydro_step(hydro_ctx *h, int32_t ncycles, void *cuda_stream, hydro_info *info) {
+  NvtxRange nvtx_("hydro_step");
   if (!h || ncycles < 0) return set_err(h, HYDRO_EINVAL, "bad argument");
   if (h->failed) return set_err(h, HYDRO_ESTATE, "context failed earlier");
   if (h->peer && !peer_ready(h->peer))
@@ -1090,6 +1099,7 @@ int hydro_domain_bytes(const hydro_ctx *h, int32_t dom, size_t *len) {
 }
 
 int hydro_domain_pack(hydro_ctx *h, int32_t dom, void *dev_buf, size_t len, void *stream) {
+  NvtxRange nvtx_("hydro_domain_pack");
   size_t need = 0;
   if (hydro_domain_bytes(h, dom, &need) || !dev_buf || len < need ||
       h->slot_of_dom[dom] < 0)
@@ -1115,6 +1125,7 @@ int hydro_domain_pack(hydro_ctx *h, int32_t dom, void *dev_buf, size_t len, void
 
 int hydro_domain_unpack(hydro_ctx *h, int32_t dom, const void *dev_buf, size_t len,
                         void *stream) {
+  NvtxRange nvtx_("hydro_domain_unpack");
   size_t need = 0;
   if (hydro_domain_bytes(h, dom, &need) || !dev_buf || len < need ||
       h->slot_of_dom[dom] < 0)
@@ -1161,6 +1172,7 @@ int hydro_set_clock(hydro_ctx *h, double t, double dt, int64_t cycle) {
 
 int hydro_get_box(hydro_ctx *h, const int64_t lo[3], const int64_t hi[3], uint32_t mask,
                   double *const *out) {
+  NvtxRange nvtx_("hydro_get_box");
   if (!h || !lo || !hi || !out) return set_err(h, HYDRO_EINVAL, "NULL argument");
   for (int a = 0; a < 3; ++a)
     if (lo[a] < 0 || hi[a] > h->L.N[a] || hi[a] <= lo[a])
@@ -1233,6 +1245,7 @@ int hydro_get_box(hydro_ctx *h, const int64_t lo[3], const int64_t hi[3], uint32
 }
 
 int hydro_get_fields(hydro_ctx *h, uint32_t mask, double *const *out) {
+  NvtxRange nvtx_("hydro_get_fields");
   if (!h) return set_err(h, HYDRO_EINVAL, "NULL context");
   const int64_t lo[3] = {0, 0, 0};
   const int64_t hi[3] = {h->L.N[0], h->L.N[1], h->L.N[2]};
@@ -1241,6 +1254,7 @@ int hydro_get_fields(hydro_ctx *h, uint32_t mask, double *const *out) {
 
 int hydro_set_state(hydro_ctx *h, const double *const *nodes6, const double *e, double t,
                     double dt) {
+  NvtxRange nvtx_("hydro_set_state");
   if (!h || !nodes6 || !e || !(dt > 0.0)) return set_err(h, HYDRO_EINVAL, "bad argument");
   for (int f = 0; f < 6; ++f)
     if (!nodes6[f]) return set_err(h, HYDRO_EINVAL, "missing node array");
@@ -1326,6 +1340,7 @@ void batch_gather(hydro_ctx *h, double *dense, int par, cudaStream_t s) {
 
 int hydro_run_batch(hydro_ctx *h, int32_t nbatch, int32_t ncycles, const double *const *in,
                     double *const *out, const double *t0, const double *dt0, hydro_info *info) {
+  NvtxRange nvtx_("hydro_run_batch");
   if (!h || nbatch < 0 || ncycles < 0 || (nbatch > 0 && (!in || !out || !t0 || !dt0)))
     return set_err(h, HYDRO_EINVAL, "run_batch: bad argument");
   if (h->cfg.nranks > 1 || h->peer || h->comm)
@@ -1464,6 +1479,7 @@ int hydro_kernels_per_cycle(const hydro_ctx *h) {
 }
 
 int hydro_time_kernels(hydro_ctx *h, int32_t ncycles, double out_ms[6]) {
+  NvtxRange nvtx_("hydro_time_kernels");
   if (!h || ncycles <= 0 || !out_ms) return set_err(h, HYDRO_EINVAL, "bad argument");
   if (h->failed) return set_err(h, HYDRO_ESTATE, "context failed earlier");
   if (h->peer && !peer_ready(h->peer))

@@ -1,3 +1,4 @@
+# (study build: git show 5ecd0f5..HEAD~0 history; needs -DHYDRO_NODE_TY_HALF=5 -DHYDRO_RACE_COSCHED, removed after the study)
 # co-scheduling study (DESIGN.md §14 lever 1): node stage at half-SM tiles (32x5, 256 threads,
 # <= 128 registers, 113 KB) next to the zone stage; HYDRO_RACE_COSCHED runs both kernels of a
 # cycle concurrently WITHOUT their dependency (timing only, results wrong)
