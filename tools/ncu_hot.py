@@ -7,7 +7,13 @@ n = int(sys.argv[4]) if len(sys.argv) > 4 else 25
 out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass",
                       "-k", "regex:" + kre], capture_output=True, text=True).stdout.splitlines()
 rows = list(csv.reader(out[1:]))
-hdr, body = rows[0], rows[1:]
+hdr = rows[0]
+body = []
+for r in rows[1:]:  # the first launch's section only (later launches repeat the listing)
+    if r and r[0] == "Kernel Name":
+        break
+    if len(r) == len(hdr):
+        body.append(r)
 ci, si, ai = hdr.index(col), hdr.index("Source"), hdr.index("Address")
 tot = sum(float(r[ci] or 0) for r in body) or 1.0
 allc = hdr.index("Warp Stall Sampling (All Samples)")
