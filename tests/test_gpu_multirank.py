@@ -103,3 +103,40 @@ def test_two_ranks_uneven_mixed_domains_match_oracle(halo):
     assert i0["status"] == 0 and i0["dt"] == i1["dt"]
     for k in FIELDS:
         assert rel_err(f[k], fo[k]) <= 1e-10, k
+
+
+def test_tangled_zone_on_one_rank_halts_both_at_the_same_cycle():
+    """ADVICE r1 / SURVEY §8b: the error bits are reduced with dt every cycle, so a zone tangled
+    in rank 1's domain halts rank 0 too, at the oracle's cycle with the oracle's status (the
+    NCCL transport reduces them the same way: one allreduce over [~dt, error words])."""
+    from tests.helpers import user_state
+    n = (8, 8, 8)
+    s = user_state(n, e=1.0)
+    s["u"][3, 6, 3] = 1e4  # node (x=3, y=6, z=3): inside the upper y-slab (rank 1)
+    kw = dict(n=n, ndom=(1, 2, 1), init="user", user=s, dt_first=1e-3)
+    i0, i1, f = run_two_ranks(kw, 5)
+    fo, io = oracle.run(OracleConfig(n=n, ndom=(1, 2, 1), init="user", user=s, dt_first=1e-3), 5)
+    assert io["status"] == -5 and io["cycle"] == 1
+    assert i0["status"] == i1["status"] == -5
+    assert i0["cycle"] == i1["cycle"] == io["cycle"]
+    assert i1["bad_zone"] == io["bad_zone"]  # the owning rank names the zone
+    # both ranks keep the state after the failing cycle (same clock as the oracle); the fields
+    # around a zone of negative volume are not comparable within a rounding tolerance (the
+    # fast reciprocals and the oracle's division diverge on V <= 0), so only the far side is
+    assert i0["t"] == i1["t"] == pytest.approx(io["t"], rel=1e-14)
+    for k in ("x", "u", "e"):
+        far = (slice(None), slice(0, 2), slice(None))  # y-planes 0-1: rank 0, far from the node
+        assert rel_err(f[k][far], fo[k][far]) <= 1e-12, k
+
+
+def test_dt_floor_halts_both_ranks_at_the_same_cycle():
+    n = (16, 16, 16)
+    s = jittered_state(n, 1)
+    o = oracle.Oracle(OracleConfig(n=n, init="user", user=s, dt_floor=-1.0))
+    seq = [o.step(1)["dt_min_zone"] for _ in range(12)]
+    o.close()
+    floor = 0.5 * (seq[9] + min(seq[:9]))
+    kw = dict(n=n, ndom=(1, 2, 1), init="user", user=s, dt_floor=floor)
+    i0, i1, f = run_two_ranks(kw, 100)
+    assert i0["status"] == i1["status"] == -7
+    assert i0["cycle"] == i1["cycle"] == 10
