@@ -79,3 +79,28 @@ def test_default_line_is_the_headline_config():
     assert d["weak384"]["value"] > 0 and d["weak384"]["workload"].startswith("weak scaling 384")
     assert d["selfcheck"]["pass"] is True
     assert d["e2e"]["h2d_bytes_per_step"] > 7e9
+
+
+@pytest.mark.parametrize("ngpu", [1, 2, 4, 8])
+def test_bench_workloads_are_the_baseline_configs(ngpu):
+    """The configurations bench.py times at N GPUs are BASELINE.json's: configs[2] = 512^3 in 8
+    domains over N GPUs (strong; every rank gets 8/N domains of equal size), configs[3] = weak
+    384^3 per GPU as 4 y-slab domains per GPU (host-only layout; no GPU needed)."""
+    import sys
+    sys.path.insert(0, ROOT)
+    import bench
+    kw, scaling, desc, h = bench.workload("sedov512", ngpu)
+    assert scaling == "strong" and desc.startswith("Sedov blast 3D 512^3")
+    nd = kw["ndom"][0] * kw["ndom"][1] * kw["ndom"][2]
+    assert nd == 8 and tuple(kw["n"]) == (512, 512, 512)
+    d2r = list(kw["dom_to_rank"])
+    assert sorted(d2r) == sorted([r for r in range(ngpu) for _ in range(8 // ngpu)])
+    for a in range(3):
+        c = list(kw["cuts"][a])
+        steps = {c[i + 1] - c[i] for i in range(len(c) - 1)}
+        assert len(steps) == 1  # equal domains
+    kw, scaling, desc, h = bench.workload("weak384", ngpu)
+    assert scaling == "weak" and abs(h - 1.2 / 384) < 1e-15
+    n = kw["n"]
+    assert n[0] * n[1] * n[2] == ngpu * 384 ** 3
+    assert kw["ndom"][0] * kw["ndom"][1] * kw["ndom"][2] == 4 * ngpu
