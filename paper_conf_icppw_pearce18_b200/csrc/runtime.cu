@@ -110,6 +110,10 @@ struct hydro_ctx {
   cudaEvent_t in_ready[2] = {}, in_free[2] = {}, out_ready[2] = {}, out_free[2] = {};
   DevState *bst = nullptr;  // per-batch final DevState
   int32_t bst_cap = 0;
+  // hydro_step early stop (single rank): a ring of pinned mirrors of (halted, done)
+  static constexpr int NFLAG = 8;
+  unsigned int *flag_host = nullptr;
+  cudaEvent_t flag_ev[NFLAG] = {};
   double *stage = nullptr;  // contiguous device staging for host transfers (lazy)
   size_t stage_cap = 0;
   std::string err;
@@ -1054,7 +1058,49 @@ int hydro_step(hydro_ctx *h, int32_t ncycles, void *cuda_stream, hydro_info *inf
     return set_err(h, HYDRO_ESTATE, "peer transport: hydro_peer_import not called yet");
   CK(cudaSetDevice(h->device));
   cudaStream_t s = cuda_stream ? (cudaStream_t)cuda_stream : h->stream;
+  // Early stop (one rank only: every rank must launch the same cycles, whose collectives pair
+  // up): once the run halted or reached t_stop, the remaining cycles are no-ops on the device
+  // (that still copy the state between parities), so stop launching them.  Every 64 cycles the
+  // (halted, done) words are copied to a ring of pinned host slots behind events; completed
+  // slots are polled without blocking, and the host is never more than NFLAG x 64 cycles ahead
+  // of the last confirmed check (it waits on the oldest slot when the ring is full), so at
+  // most ~NFLAG x 64 no-op cycles run past the end.
+  const bool early = h->cfg.nranks <= 1;
+  constexpr int NF = hydro_ctx::NFLAG;
+  if (early && !h->flag_host) {
+    CK(cudaHostAlloc(&h->flag_host, 2 * NF * sizeof(unsigned int), cudaHostAllocDefault));
+    for (int k = 0; k < NF; ++k)
+      CK(cudaEventCreateWithFlags(&h->flag_ev[k], cudaEventDisableTiming));
+  }
+  int oldest = 0, npend = 0;
+  int32_t next_check = 64;
+  bool stop = false;
+  auto pop_done = [&](bool block) -> cudaError_t {  // true in `stop` when a slot shows the end
+    while (npend > 0) {
+      cudaError_t q = block ? cudaEventSynchronize(h->flag_ev[oldest])
+                            : cudaEventQuery(h->flag_ev[oldest]);
+      if (q == cudaErrorNotReady) return cudaSuccess;
+      if (q != cudaSuccess) return q;
+      if ((h->flag_host[2 * oldest] | h->flag_host[2 * oldest + 1]) != 0u) stop = true;
+      oldest = (oldest + 1) % NF;
+      --npend;
+      block = false;
+      if (stop) return cudaSuccess;
+    }
+    return cudaSuccess;
+  };
   for (int32_t c = 0; c < ncycles;) {
+    if (early && c >= next_check) {
+      next_check = c + 64;
+      CK(pop_done(false));
+      if (!stop && npend == NF) CK(pop_done(true));
+      if (stop) break;
+      const int slot = (oldest + npend) % NF;
+      CK(cudaMemcpyAsync(&h->flag_host[2 * slot], &h->st->halted, 2 * sizeof(unsigned int),
+                         cudaMemcpyDeviceToHost, s));
+      CK(cudaEventRecord(h->flag_ev[slot], s));
+      ++npend;
+    }
     if (h->use_graph && h->graph_k > 1 && ncycles - c >= h->graph_k) {
       CK(cudaGraphLaunch(h->graphk[h->parity], s));
       h->parity ^= h->graph_k & 1;
@@ -1558,6 +1604,9 @@ int hydro_destroy(hydro_ctx *h) {
   if (!h) return HYDRO_OK;
   cudaSetDevice(h->device);
   if (h->stream) cudaStreamSynchronize(h->stream);
+  for (int k = 0; k < hydro_ctx::NFLAG; ++k)
+    if (h->flag_ev[k]) cudaEventDestroy(h->flag_ev[k]);
+  if (h->flag_host) cudaFreeHost(h->flag_host);
   if (h->pcopy_dev) cudaFree(h->pcopy_dev);
   for (int p = 0; p < 2; ++p) {
     if (h->graph[p]) cudaGraphExecDestroy(h->graph[p]);
