@@ -150,7 +150,11 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out);
    context's own stream) and the call returns after it completed (one host synchronisation per
    call, not per cycle).  info (optional) receives the state after the last cycle.  Collective.
    Returns HYDRO_OK, or the physics error of the cycle that failed (the state is the one after
-   that cycle; later calls return HYDRO_ESTATE), or HYDRO_ECUDA / HYDRO_ENCCL. */
+   that cycle; later calls return HYDRO_ESTATE), or HYDRO_ECUDA / HYDRO_ENCCL.  Cycles after
+   t_stop or after a failure are no-ops; a single-rank context stops launching them (within
+   ~512 cycles of the end), a multi-rank one launches all of them (their collectives pair up
+   across ranks).  HYDRO_ENCCL also covers an NCCL asynchronous error or a wait longer than
+   HYDRO_NCCL_TIMEOUT_S seconds (default 600): the communicators are then aborted. */
 int hydro_step(hydro_ctx *h, int32_t ncycles, void *cuda_stream, hydro_info *info);
 
 /* Copy fields of the current state into caller-owned global host arrays.  out[f] is used for
