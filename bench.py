@@ -159,9 +159,10 @@ def fp64_peak():
 
 
 def kernel_counters():
-    """Per-kernel ncu counters at 128^3 (profiles/kernel_counters.json, written by
-    tools/ncu_summary.py from an `ncu --set full` capture): DRAM bytes per owned
-    zone and executed fp64 pipe instructions (DADD+DMUL+DFMA, thread level) per owned zone."""
+    """Per-kernel ncu counters at the headline config, 512^3 in 8 domains
+    (profiles/kernel_counters.json, written by tools/ncu_summary.py from `ncu --set full`
+    captures): DRAM bytes per owned zone and executed fp64 pipe instructions
+    (DADD+DMUL+DFMA, thread level) per owned zone."""
     try:
         with open(os.path.join(ROOT, "profiles", "kernel_counters.json")) as f:
             return json.load(f)["kernels"]
@@ -371,9 +372,9 @@ class Run:
                 alu = flops / (kms * 1e-3)
                 r.update({"fp64_inst_per_s": alu, "fp64_frac": alu / fp64_peak()})
             c = KC.get(name)
-            if c:  # the same kernel under ncu at 128^3 (profiles/kernel_counters.json)
-                r["ncu_128"] = {k: c.get(k) for k in ("fp64_pipe_pct", "smem_wavefronts_pct",
-                                                      "issue_active", "dram_bytes_per_zone")}
+            if c:  # the same kernel under ncu at 512^3 (profiles/kernel_counters.json)
+                r["ncu"] = {k: c.get(k) for k in ("fp64_pipe_pct", "smem_wavefronts_pct",
+                                                  "issue_active", "dram_bytes_per_zone")}
             rows.append(r)
         dom = max(rows, key=lambda r: r["ms"])
         alu_bound = dom.get("fp64_frac", 0.0) > dom["hbm_frac"]
@@ -384,7 +385,7 @@ class Run:
                 "frac": dom["fp64_frac"] if alu_bound else dom["hbm_frac"],
                 "traffic": (TRAFFIC_PER_ZONE[dom["kernel"]] * Nz
                             if TRAFFIC_PER_ZONE.get(dom["kernel"]) else None),
-                "traffic_source": "ncu dram__bytes_read+write per zone at 128^3 "
+                "traffic_source": "ncu dram__bytes_read+write per zone at 512^3 / 8 domains "
                                   "(profiles/kernel_counters.json) x this launch's zones",
                 "peak_source": ("measured DFMA rate (profiles/r01_fp64_peak.txt)" if alu_bound
                                 else f"{peak_kind} MEASURED_PEAKS.json hbm_gbs"),
@@ -515,27 +516,24 @@ def selfcheck(args, name, ngpu, rank, local, dist):
 def nccl_leg(args, name, ngpu, rank, local, dist, share):
     """N>1 with the peer transport: 10 cycles of the same configuration with the NCCL transport
     (grouped send/recv halo + allreduce), compared bitwise with the peer run per local domain
-    (hydro_domain_pack), so a multi-GPU driver run executes comm.cu."""
+    (hydro_domain_pack), so a multi-GPU driver run executes comm.cu.  A failure is reported in
+    the line (the timed numbers stand); a stalled NCCL leg ends in HYDRO_ENCCL after
+    HYDRO_NCCL_TIMEOUT_S (set to 120 s here; comm_wait polls ncclCommGetAsyncError)."""
     if ngpu < 2 or args.transport != "peer":
         return None
     if share:
         return {"ran": False, "why": "ranks share one GPU (HYDRO_SHARE_GPU): NCCL refuses"}
-    import torch
-    from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig, dom_to_rank
-    # a stalled NCCL leg ends in HYDRO_ENCCL after this long (comm_wait polls
-    # ncclCommGetAsyncError), not in a hung bench
     os.environ.setdefault("HYDRO_NCCL_TIMEOUT_S", "120")
-    kw, _, _, _ = workload(name, ngpu)
-    packs, ms = {}, {}
     try:
-        return _nccl_leg_run(args, kw, ngpu, rank, local, dist, torch, Hydro, HydroConfig,
-                             dom_to_rank, packs, ms)
-    except Exception as exc:  # reported in the line, the timed numbers above stand
+        return _nccl_vs_peer(args, workload(name, ngpu)[0], ngpu, rank, local, dist)
+    except Exception as exc:
         return {"ran": True, "error": f"{type(exc).__name__}: {exc}"[:300]}
 
 
-def _nccl_leg_run(args, kw, ngpu, rank, local, dist, torch, Hydro, HydroConfig, dom_to_rank,
-                  packs, ms):
+def _nccl_vs_peer(args, kw, ngpu, rank, local, dist):
+    import torch
+    from paper_conf_icppw_pearce18_b200 import Hydro, HydroConfig, dom_to_rank
+    packs, infos, ms = {}, {}, {}
     for tr in ("peer", "nccl"):
         cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, path=args.path, transport=tr,
                           hg_coef=args.hg, halo=args.halo, **kw)
@@ -544,14 +542,14 @@ def _nccl_leg_run(args, kw, ngpu, rank, local, dist, torch, Hydro, HydroConfig, 
         torch.cuda.synchronize()
         dist.barrier()
         t0 = time.perf_counter()
-        info = hyd.step(10)
+        infos[tr] = hyd.step(10)
         ms[tr] = (time.perf_counter() - t0) * 1e3 / 10
         mine = [d for d, r in enumerate(dom_to_rank(cfg)) if r == rank]
-        packs[tr] = ({d: hyd.pack_domain(d).cpu() for d in mine}, info)
+        packs[tr] = {d: hyd.pack_domain(d).cpu() for d in mine}
         hyd.close()
-    same = all(torch.equal(packs["peer"][0][d], packs["nccl"][0][d]) for d in packs["peer"][0])
-    same_t = packs["peer"][1]["t"] == packs["nccl"][1]["t"]
-    flag = torch.tensor([1.0 if (same and same_t) else 0.0], device="cuda")
+    same = all(torch.equal(packs["peer"][d], packs["nccl"][d]) for d in packs["peer"])
+    same = same and infos["peer"]["t"] == infos["nccl"]["t"]
+    flag = torch.tensor([1.0 if same else 0.0], device="cuda")
     dist.all_reduce(flag, op=dist.ReduceOp.MIN)
     return {"ran": True, "cycles": 12, "bitwise_equal_to_peer": bool(flag.item() == 1.0),
             "wall_ms_per_cycle": ms, "transport": "nccl (ncclSend/ncclRecv group + allreduce)"}
