@@ -361,7 +361,7 @@ class Run:
         elif args.path == "one":
             kern.append(("k_cycle_fused", kt["cycle_kernel_ms"], 96.0 * Nn + 24.0 * Nz, None))
         else:
-            kern.append(("split zone+node+energy", kt["cycle_kernel_ms"],
+            kern.append((f"{args.path} zone+node+energy", kt["cycle_kernel_ms"],
                          96.0 * Nn + 24.0 * Nz, None))
         rows = []
         for name, kms, byts, flops in kern:
@@ -564,8 +564,9 @@ def main():
     ap.add_argument("--second", default="weak384",
                     help="second configuration timed in the same run ('' = none)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--path", default="two", choices=["two", "one", "split"],
-                    help="two: zone + node/energy kernels; one: one fused kernel; split: plain")
+    ap.add_argument("--path", default="two", choices=["two", "one", "split", "strict"],
+                    help="two: zone + node/energy kernels; one: one fused kernel; split: plain; "
+                         "strict: the split pipeline in the oracle's order without FMA (bitwise)")
     ap.add_argument("--transport", default="peer", choices=["peer", "nccl"],
                     help="N>1 halo/dt transport: CUDA IPC peer stores or NCCL send/recv + "
                          "allreduce (the other one is run as a 10-cycle bitwise check)")

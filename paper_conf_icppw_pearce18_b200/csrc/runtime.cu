@@ -957,7 +957,7 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
          if (cfg->nranks > 1 && (cfg->flags & HYDRO_FLAG_PEER)) {
            int r = peer_create(&h->peer, cfg, &h->err);
            if (r) return r;
-         } else if (cfg->nranks > 1) {
+         } else if (cfg->nranks > 1 || (cfg->flags & HYDRO_FLAG_COMM_SELF)) {
            int r = comm_create(&h->comm, cfg, h->L, remote, h->slot_of_dom, h->doms.empty() ? nullptr : nullptr,
                                h->stream, &h->err);
            if (r) return r;

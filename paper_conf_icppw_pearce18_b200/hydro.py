@@ -29,6 +29,7 @@ FLAG_ONE_KERNEL = 1 << 2
 FLAG_PEER = 1 << 3
 FLAG_HALO_FUSED = 1 << 4
 FLAG_STRICT = 1 << 5
+FLAG_COMM_SELF = 1 << 6
 
 STATUS = {0: "ok", -1: "EINVAL", -2: "ENOMEM", -3: "ECUDA", -4: "ENCCL", -5: "ETANGLED",
           -6: "ENONFINITE", -7: "EDTMIN", -8: "ESTATE"}
@@ -167,6 +168,8 @@ class HydroConfig:
                                   # the split kernels
     dt_floor: float = 0.0         # dt-collapse floor (reading R23): > 0 absolute, 0 = 1e-6 dt^0,
                                   # < 0 none; below it a run halts with EDTMIN
+    comm_self: bool = False       # nranks == 1: create a one-rank NCCL communicator anyway
+                                  # (HYDRO_FLAG_COMM_SELF; exercises the NCCL path on one GPU)
 
 
 class HydroError(RuntimeError):
@@ -215,6 +218,7 @@ def _cfg_struct(cfg: HydroConfig, keep: list, comm_id: Optional[bytes] = None) -
     c.flags = ((0 if cfg.graph else FLAG_NO_GRAPH) | (FLAG_SPLIT if cfg.path == "split" else 0)
                | (FLAG_ONE_KERNEL if cfg.path == "one" else 0)
                | (FLAG_STRICT if cfg.path == "strict" else 0)
+               | (FLAG_COMM_SELF if cfg.comm_self else 0)
                | (FLAG_PEER if cfg.transport == "peer" else 0)
                | (FLAG_HALO_FUSED if cfg.halo == "fused" else 0))
     return c
@@ -325,6 +329,12 @@ class Hydro:
         comm_id = None
         if cfg.nranks > 1 and cfg.transport == "nccl":
             comm_id = self._bootstrap_comm_id()
+        elif cfg.comm_self:  # one-rank NCCL world (testing the NCCL path on one GPU)
+            raw = C.create_string_buffer(128)
+            rc = self._L.hydro_comm_unique_id(raw)
+            if rc != 0:
+                raise HydroError(rc, "hydro_comm_unique_id")
+            comm_id = raw.raw
         keep: list = []
         c = _cfg_struct(cfg, keep, comm_id)
         h = C.c_void_p()
