@@ -78,10 +78,14 @@ enum {
                                              kernels after it (correct, measured
                                              slower on B200, so opt-in) */
 #define HYDRO_FLAG_COMM_SELF (1ull << 6) /* nranks == 1: still create the NCCL communicator
-                                             (a one-rank world; comm_id required), so the NCCL
-                                             dt / error allreduce, its overlap stream, the async-
-                                             error polling and the teardown run on a one-GPU box
-                                             (testing; results equal the communicator-free run) */
+                                             (a one-rank world; comm_id required) and move the
+                                             ghost slabs between this rank's domains by NCCL
+                                             send/recv to itself (pack, grouped send/recv,
+                                             unpack) instead of the copy kernel, so the NCCL
+                                             halo and dt / error allreduce, its overlap stream,
+                                             the async-error polling and the teardown run on a
+                                             one-GPU box (testing; results equal the
+                                             communicator-free run bitwise) */
 #define HYDRO_FLAG_STRICT (1ull << 5)     /* the split pipeline evaluated in the canonical
                                              operation order of SURVEY §8c (readings R12, R13),
                                              compiled without FMA contraction: BITWISE equal to

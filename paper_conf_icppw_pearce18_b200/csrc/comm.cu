@@ -107,7 +107,7 @@ int comm_create(Comm **out, const hydro_config *cfg, const Layout &L,
     return HYDRO_ENCCL;
   }
   std::vector<PlanEntry> snd, rcv;
-  comm_plan(L, cfg->rank, &snd, &rcv);
+  comm_plan(L, cfg->rank, &snd, &rcv, (cfg->flags & HYDRO_FLAG_COMM_SELF) != 0);
   (void)remote;
   for (int dir = 0; dir < 2; ++dir) {
     for (const PlanEntry &e : dir ? rcv : snd) {

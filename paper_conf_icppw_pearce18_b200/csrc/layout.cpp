@@ -165,13 +165,13 @@ std::vector<int64_t> layout_serialise(const Layout &L) {
 }
 
 void comm_plan(const Layout &L, int32_t rank, std::vector<PlanEntry> *sends,
-               std::vector<PlanEntry> *recvs) {
+               std::vector<PlanEntry> *recvs, bool self_all) {
   sends->clear();
   recvs->clear();
   for (size_t i = 0; i < L.pairs.size(); ++i) {
     const HaloPair &P = L.pairs[i];
     const int32_t rd = L.dom[P.dst].rank, rs = L.dom[P.src].rank;
-    if (rd == rs) continue;  // same rank: intra-GPU copy kernel
+    if (rd == rs && !(self_all && rd == rank)) continue;  // same rank: intra-GPU copy kernel
     int64_t nn = 1, nz = 1;
     for (int a = 0; a < 3; ++a) {
       nn *= P.nhi[a] - P.nlo[a];

@@ -57,7 +57,9 @@ struct PlanEntry {
   int32_t peer;   // remote rank
   int64_t count;  // doubles: 6 node fields over the node slab + e over the zone slab
 };
+// self_all: also plan the pairs whose two domains are on this rank (as messages to itself;
+// the one-rank NCCL test world, HYDRO_FLAG_COMM_SELF)
 void comm_plan(const Layout &L, int32_t rank, std::vector<PlanEntry> *sends,
-               std::vector<PlanEntry> *recvs);
+               std::vector<PlanEntry> *recvs, bool self_all = false);
 
 }  // namespace hydro

@@ -838,6 +838,9 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
          }
          std::vector<HaloCopy> lp, pc;
          std::vector<HaloPair> remote;
+         // HYDRO_FLAG_COMM_SELF: the same-rank ghost slabs go through NCCL self send/recv
+         // (comm_plan self_all) instead of the intra-GPU copy; only their P copies stay
+         const bool self_halo = (cfg->flags & HYDRO_FLAG_COMM_SELF) != 0;
          for (const HaloPair &P : h->L.pairs) {
            const bool dst_local = h->slot_of_dom[P.dst] >= 0;
            const bool src_local = h->slot_of_dom[P.src] >= 0;
@@ -865,6 +868,7 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
              // once more for P when the destination's zone stage skips its ring there
              for (int kind = 0; kind < 3; ++kind) {
                if (kind == 2 && h->ring[c.dst] == 0x3f) continue;
+               if (kind < 2 && self_halo) continue;
                const int64_t total = kind ? nz : nn;
                for (int64_t st = 0; st < total; st += HALO_CHUNK) {
                  c.kind = kind;

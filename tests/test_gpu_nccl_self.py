@@ -1,11 +1,14 @@
 """The NCCL transport's device-side plumbing on the pool's single B200: a one-rank NCCL world
-(HYDRO_FLAG_COMM_SELF).  Every cycle then runs the NCCL dt / error allreduce (pack, allreduce
-over [~dt, error words], unpack), on its own communicator (ncclCommSplit) and stream forked
-after the zone stage and joined before S9 (two-kernel path) or in line (other paths), captured
-in the CUDA graphs; hydro_step waits while polling ncclCommGetAsyncError.  With one rank the
-reduction is the identity, so every field, t and dt must equal the communicator-free run bit for
-bit, including a run that halts with EDTMIN.  (Two ranks on one GPU are refused by NCCL, so the
-grouped send/recv halo leg runs only on multi-GPU nodes: bench.py's nccl_check.)"""
+(HYDRO_FLAG_COMM_SELF).  Every cycle then moves the ghost slabs between the rank's domains by
+the NCCL halo leg (pack kernel, grouped ncclSend/ncclRecv to itself in plan order, unpack
+kernel) instead of the copy kernel, and runs the NCCL dt / error allreduce (pack, allreduce over
+[~dt, error words], unpack) on its own communicator (ncclCommSplit) and stream, forked after the
+zone stage and joined before S9 (two-kernel path) or in line (other paths), all captured in the
+CUDA graphs; hydro_step waits while polling ncclCommGetAsyncError.  The slabs are bit copies
+and the one-rank reduction is the identity, so every field, t and dt must equal the
+communicator-free run bit for bit, including a run that halts with EDTMIN.  (NCCL refuses two
+ranks on one GPU; the cross-rank plan matching is covered by the gloo tests and bench.py's
+nccl_check at N > 1.)"""
 import numpy as np
 import pytest
 
@@ -21,6 +24,7 @@ def _run(nc, **kw):
     with Hydro(HydroConfig(**kw)) as h:
         info = h.step(nc)
         f = h.fields()
+        info["kernels"] = h.kernels_per_cycle()
     return f, info
 
 
@@ -34,6 +38,7 @@ def test_one_rank_nccl_equals_no_comm_bitwise(path, overlap, monkeypatch):
     fb, ib = _run(30, **kw)
     assert ia["status"] == ib["status"] == 0
     assert ia["t"] == ib["t"] and ia["dt"] == ib["dt"] and ia["cycle"] == ib["cycle"] == 30
+    assert ia["kernels"] != ib["kernels"]  # pack / unpack / dt kernels instead of the copies
     for k in FIELDS:
         assert np.array_equal(fa[k], fb[k]), k
 
