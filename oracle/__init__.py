@@ -52,6 +52,10 @@ def lib() -> C.CDLL:
         L.orc_zone_state.restype = None
         L.orc_zone_hourglass.argtypes = [C.c_void_p] * 3 + [C.c_double] * 4 + [C.c_void_p]
         L.orc_zone_hourglass.restype = None
+        L.orc_zone_strain.argtypes = [C.c_void_p] * 4
+        L.orc_zone_strain.restype = None
+        L.orc_mono_limiter.argtypes = [C.c_double] * 3
+        L.orc_mono_limiter.restype = C.c_double
         _lib = L
     return _lib
 
@@ -73,6 +77,7 @@ class _Config(C.Structure):
         ("user", C.POINTER(C.c_double) * 8),
         ("hg_coef", C.c_double),
         ("dt_floor", C.c_double),
+        ("q_kind", C.c_int32),
     ]
 
 
@@ -111,6 +116,7 @@ class OracleConfig:
     user: Optional[Dict[str, np.ndarray]] = None
     hg_coef: float = 0.0                  # reading R17 / SURVEY §8f f1: hourglass kappa, 0 = off
     dt_floor: float = 0.0                 # reading R23: > 0 absolute, 0 = 1e-6 dt^0, < 0 none
+    q: str = "scalar"                     # "scalar" (reading R7) | "monotone" (reading R24)
 
 
 class OracleError(RuntimeError):
@@ -143,6 +149,7 @@ class Oracle:
             setattr(c, k, float(getattr(cfg, k)))
         c.reflect_mask = int(cfg.reflect_mask)
         c.init_kind = INIT[cfg.init]
+        c.q_kind = {"scalar": 0, "monotone": 1}[cfg.q]
         if cfg.init != "sedov":
             names = ("x", "y", "z", "u", "v", "w", "rho" if cfg.init == "user" else "mass", "e")
             for f, nm in enumerate(names):
@@ -232,6 +239,20 @@ def zone_hourglass(X, U, B, V, rho, c, kappa) -> np.ndarray:
     lib().orc_zone_hourglass(X.ctypes.data, U.ctypes.data, B.ctypes.data, float(V), float(rho),
                              float(c), float(kappa), F.ctypes.data)
     return F
+
+
+def zone_strain(X, U):
+    """Reading R24: (eps (3,), L (3,)) of one zone (orc_zone_strain)."""
+    X = np.ascontiguousarray(X, dtype=np.float64).reshape(8, 3)
+    U = np.ascontiguousarray(U, dtype=np.float64).reshape(8, 3)
+    eps, L = np.zeros(3), np.zeros(3)
+    lib().orc_zone_strain(X.ctypes.data, U.ctypes.data, eps.ctypes.data, L.ctypes.data)
+    return eps, L
+
+
+def mono_limiter(em, e0, ep) -> float:
+    """Reading R24: the monotonic limiter phi of one direction (orc_mono_limiter)."""
+    return float(lib().orc_mono_limiter(float(em), float(e0), float(ep)))
 
 
 def run(cfg: OracleConfig, ncycles: int, names: Sequence[str] = ALL_FIELDS):

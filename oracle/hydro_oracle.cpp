@@ -94,7 +94,48 @@ void geometry(const double X[8][3], double B[8][3], double *V, double *L) {
 struct Params {
   double gamma, gm1, ggm1, q_lin, q_quad, cfl, c_vol;
   double hg;  // hourglass coefficient kappa (reading R17; 0 = off)
+  int q_kind = 0;  // 0 scalar q (reading R7), 1 monotone q (reading R24)
 };
+
+// f1 / reading R24: the zone's strain rate along each logical direction d (0 = xi, 1 = eta,
+// 2 = zeta): face-centre differences dx_d = (mean of the 4 corners with bit d = 1) - (mean with
+// bit d = 0), du_d likewise for the velocities (corner sums in ascending l, first term
+// initialising); L_d = |dx_d|; eps_d = (du_d . dx_d) / (dx_d . dx_d).
+void strain(const double X[8][3], const double U[8][3], double eps[3], double L[3]) {
+  for (int d = 0; d < 3; ++d) {
+    double xs[2][3], us[2][3];
+    bool first[2] = {true, true};
+    for (int l = 0; l < 8; ++l) {
+      const int side = (l >> d) & 1;
+      for (int k = 0; k < 3; ++k) {
+        xs[side][k] = first[side] ? X[l][k] : xs[side][k] + X[l][k];
+        us[side][k] = first[side] ? U[l][k] : us[side][k] + U[l][k];
+      }
+      first[side] = false;
+    }
+    double dx[3], du[3];
+    for (int k = 0; k < 3; ++k) {
+      dx[k] = 0.25 * (xs[1][k] - xs[0][k]);
+      du[k] = 0.25 * (us[1][k] - us[0][k]);
+    }
+    const double L2 = dot3(dx, dx);
+    eps[d] = dot3(du, dx) / L2;
+    L[d] = std::sqrt(L2);
+  }
+}
+
+// Reading R24: monotonic limiter of direction d from the strain rates of the zone (e0) and of its
+// two neighbours along d (em, ep): phi = max(0, min(1/2 (rm + rp), 2 rm, 2 rp, 1)) with
+// r = e_neighbour / e0 (the MC-type limiter of Christensen / LULESH); phi = 1 when e0 = 0.
+double mono_limiter(double em, double e0, double ep) {
+  if (e0 == 0.0) return 1.0;
+  const double rm = em / e0, rp = ep / e0;
+  double phi = 0.5 * (rm + rp);
+  phi = std::min(phi, 2.0 * rm);
+  phi = std::min(phi, 2.0 * rp);
+  phi = std::min(phi, 1.0);
+  return std::max(phi, 0.0);
+}
 
 struct ZoneOut {
   double rho, ep, p, c, q, P, dtz, V, L, D;
@@ -102,8 +143,9 @@ struct ZoneOut {
 
 // S2 (DV, rho, D) + S3 (predictor, EOS) + S4 (q, P) + S6 (dt_z) for one zone
 // (readings R5-R8).  X are the half-step positions x_p, U the velocities u^n.
+// phi (reading R24, q_kind 1): the zone's three limiter values; nullptr for the scalar q.
 void zone_state(const double X[8][3], const double U[8][3], double m, double e, double hh,
-                const Params &pr, double B[8][3], ZoneOut *o) {
+                const Params &pr, double B[8][3], ZoneOut *o, const double *phi = nullptr) {
   double V, L;
   geometry(X, B, &V, &L);
   double DV = 0.0;
@@ -123,9 +165,18 @@ void zone_state(const double X[8][3], const double U[8][3], double m, double e, 
   const double c = std::sqrt(pr.ggm1 * eppos);
   // S4
   double qr = 0.0;
-  if (D < 0.0) {
+  if (D < 0.0 && !phi) {
     const double s = L * (-D);
     qr = s * ((pr.q_quad * s) + (pr.q_lin * c));
+  } else if (D < 0.0) {  // reading R24: per direction, limited by the neighbours' strain rates
+    double eps[3], Ld[3];
+    strain(X, U, eps, Ld);
+    for (int d = 0; d < 3; ++d) {
+      const double dv = Ld[d] * std::max(-eps[d], 0.0);
+      const double t = ((pr.q_quad * dv) * dv) * (1.0 - phi[d] * phi[d]) +
+                       ((pr.q_lin * c) * dv) * (1.0 - phi[d]);
+      qr = (d == 0) ? t : qr + t;
+    }
   }
   const double q = rho * qr;
   const double P = p + q;
@@ -227,6 +278,7 @@ struct Domain {
   std::vector<double> x[3], u[3], xn[3], un[3], xp[3], uh[3];
   std::vector<double> m, e, en, P, B;  // B: 24 per zone
   std::vector<double> HG;              // hourglass corner forces, 24 per zone (kappa > 0 only)
+  std::vector<double> eps[3];          // strain rates of the owned zones (monotone q only, R24)
   std::vector<uint8_t> zex, nex;       // exists in the global mesh
 
   int64_t zid(int64_t i, int64_t j, int64_t k) const {
@@ -406,6 +458,46 @@ void fail(orc_ctx *h, int code, int64_t zone) {
   if (zone >= 0 && (h->bad_zone < 0 || zone < h->bad_zone)) h->bad_zone = zone;
 }
 
+// Reading R24: the strain rates eps_d of every domain's owned zones at positions (x^n or x_p)
+// and velocities u^n.  Neighbour values are then read from the owning domain by global index,
+// so a ghost-ring zone's limiter sees exactly what its owner's does (decomposition-invariant).
+void strain_pass(const orc_ctx *h, bool half_step) {
+  for (const Domain &Dc : h->dom) {
+    Domain &D = const_cast<Domain &>(Dc);  // a per-pass cache, also filled by get_fields
+    const size_t tot_z = D.zex.size();
+    for (int d = 0; d < 3; ++d) D.eps[d].assign(tot_z, 0.0);
+    for (int64_t k = 0; k < D.n[2]; ++k)
+      for (int64_t j = 0; j < D.n[1]; ++j)
+        for (int64_t i = 0; i < D.n[0]; ++i) {
+          double X[8][3], U[8][3], eps[3], L[3];
+          gather_corners(D, half_step ? D.xp : D.x, D.u, i, j, k, X, U);
+          strain(X, U, eps, L);
+          for (int d = 0; d < 3; ++d) D.eps[d][D.zid(i, j, k)] = eps[d];
+        }
+  }
+}
+
+double eps_global(const orc_ctx *h, const int64_t g[3], int d) {
+  const Domain &S = h->dom[h->dom_index(h->zown[0][g[0]], h->zown[1][g[1]], h->zown[2][g[2]])];
+  return S.eps[d][S.zid(g[0] - S.lo[0], g[1] - S.lo[1], g[2] - S.lo[2])];
+}
+
+// Reading R24: limiter values of global zone g.  A neighbour outside the mesh mirrors the zone
+// at a reflecting wall (ratio 1) and has zero strain at a free boundary.
+void mono_phi(const orc_ctx *h, const int64_t g[3], double phi[3]) {
+  for (int d = 0; d < 3; ++d) {
+    const double e0 = eps_global(h, g, d);
+    int64_t gm[3] = {g[0], g[1], g[2]}, gp[3] = {g[0], g[1], g[2]};
+    gm[d] -= 1;
+    gp[d] += 1;
+    const double em = exists_zone(h, gm) ? eps_global(h, gm, d)
+                      : ((h->cfg.reflect_mask >> (2 * d)) & 1u) ? e0 : 0.0;
+    const double ep = exists_zone(h, gp) ? eps_global(h, gp, d)
+                      : ((h->cfg.reflect_mask >> (2 * d + 1)) & 1u) ? e0 : 0.0;
+    phi[d] = mono_limiter(em, e0, ep);
+  }
+}
+
 // One cycle S1..S9 over all domains, then the ghost exchange.
 void cycle(orc_ctx *h) {
   const double dt = h->dt;
@@ -420,6 +512,7 @@ void cycle(orc_ctx *h) {
       for (int d = 0; d < 3; ++d) D.xp[d][id] = D.x[d][id] + hh * D.u[d][id];
     }
   }
+  if (h->pr.q_kind == 1) strain_pass(h, true);  // R24: strain rates at the half step
   // S2-S6 for every existing local zone (owned and ghost); dt_z over owned zones.
   for (Domain &D : h->dom) {
     for (int64_t k = -1; k <= D.n[2]; ++k)
@@ -427,10 +520,15 @@ void cycle(orc_ctx *h) {
         for (int64_t i = -1; i <= D.n[0]; ++i) {
           const int64_t id = D.zid(i, j, k);
           if (!D.zex[id]) continue;
-          double X[8][3], U[8][3], B[8][3];
+          double X[8][3], U[8][3], B[8][3], phi[3];
           ZoneOut o;
           gather_corners(D, D.xp, D.u, i, j, k, X, U);
-          zone_state(X, U, D.m[id], D.e[id], hh, h->pr, B, &o);
+          if (h->pr.q_kind == 1) {
+            const int64_t gg[3] = {D.lo[0] + i, D.lo[1] + j, D.lo[2] + k};
+            mono_phi(h, gg, phi);
+          }
+          zone_state(X, U, D.m[id], D.e[id], hh, h->pr, B, &o,
+                     h->pr.q_kind == 1 ? phi : nullptr);
           std::memcpy(&D.B[id * 24], B, sizeof(B));
           D.P[id] = o.P;  // S5 f_l = P*B_l is formed where it is used (same bits)
           if (h->pr.hg > 0.0) {  // f1: f_l = P*B_l + f_hg_l
@@ -542,7 +640,8 @@ bool valid_config(const orc_config *c) {
     }
   }
   if (!(c->gamma > 1.0) || c->q_lin < 0.0 || c->q_quad < 0.0 || !(c->cfl > 0.0) ||
-      !(c->c_vol > 0.0) || !(c->dt_growth > 0.0) || !(c->dt_max > 0.0) || !(c->hg_coef >= 0.0))
+      !(c->c_vol > 0.0) || !(c->dt_growth > 0.0) || !(c->dt_max > 0.0) || !(c->hg_coef >= 0.0) ||
+      c->q_kind < 0 || c->q_kind > 1)
     return false;
   if (c->init_kind != ORC_INIT_SEDOV) {
     for (int f = 0; f < 8; ++f)
@@ -556,6 +655,12 @@ bool valid_config(const orc_config *c) {
 extern "C" {
 
 const char *orc_last_error(void) { return g_err.c_str(); }
+
+void orc_zone_strain(const double X[8][3], const double U[8][3], double eps[3], double L[3]) {
+  strain(X, U, eps, L);
+}
+
+double orc_mono_limiter(double em, double e0, double ep) { return mono_limiter(em, e0, ep); }
 
 void orc_zone_hourglass(const double X[8][3], const double U[8][3], const double B[8][3],
                         double V, double rho, double c, double kappa, double F[8][3]) {
@@ -617,7 +722,7 @@ int orc_create(const orc_config *cfg, orc_ctx **out) {
   h->ndy = cfg->ndom[1];
   h->ndz = cfg->ndom[2];
   h->pr = Params{cfg->gamma, cfg->gamma - 1.0, cfg->gamma * (cfg->gamma - 1.0), cfg->q_lin,
-                 cfg->q_quad, cfg->cfl, cfg->c_vol, cfg->hg_coef};
+                 cfg->q_quad, cfg->cfl, cfg->c_vol, cfg->hg_coef, cfg->q_kind};
   h->dom.resize((size_t)h->ndx * h->ndy * h->ndz);
   for (int c = 0; c < h->ndz; ++c)
     for (int b = 0; b < h->ndy; ++b)
@@ -634,15 +739,21 @@ int orc_create(const orc_config *cfg, orc_ctx **out) {
       }
   // dt^0: S2-S6 at x^0, e^0 with no predictor.
   double dtmin = INF;
+  if (h->pr.q_kind == 1) strain_pass(h, false);
   for (Domain &D : h->dom)
     for (int64_t k = 0; k < D.n[2]; ++k)
       for (int64_t j = 0; j < D.n[1]; ++j)
         for (int64_t i = 0; i < D.n[0]; ++i) {
           const int64_t id = D.zid(i, j, k);
-          double X[8][3], U[8][3], B[8][3];
+          double X[8][3], U[8][3], B[8][3], phi[3];
           ZoneOut o;
           gather_corners(D, D.x, D.u, i, j, k, X, U);
-          zone_state(X, U, D.m[id], D.e[id], 0.0, h->pr, B, &o);
+          if (h->pr.q_kind == 1) {
+            const int64_t gg[3] = {D.lo[0] + i, D.lo[1] + j, D.lo[2] + k};
+            mono_phi(h, gg, phi);
+          }
+          zone_state(X, U, D.m[id], D.e[id], 0.0, h->pr, B, &o,
+                     h->pr.q_kind == 1 ? phi : nullptr);
           dtmin = std::min(dtmin, o.dtz);
           if (!(o.V > 0.0)) {
             const int64_t g[3] = {D.lo[0] + i, D.lo[1] + j, D.lo[2] + k};
@@ -696,6 +807,7 @@ int orc_info_get(const orc_ctx *h, orc_info *info) {
 // e_p = e (hh = 0); e; m.
 int orc_get_fields(const orc_ctx *h, uint32_t mask, double *const *out) {
   if (!h || !out) return ORC_EINVAL;
+  if (h->pr.q_kind == 1) strain_pass(h, false);  // R24 limiter inputs at (x, u)
   for (size_t di = 0; di < h->dom.size(); ++di) {
     const Domain &D = h->dom[di];
     for (int64_t k = 0; k <= D.n[2]; ++k)
@@ -715,10 +827,12 @@ int orc_get_fields(const orc_ctx *h, uint32_t mask, double *const *out) {
         for (int64_t i = 0; i < D.n[0]; ++i) {
           const int64_t g[3] = {D.lo[0] + i, D.lo[1] + j, D.lo[2] + k};
           const int64_t gi = gzone(h, g), id = D.zid(i, j, k);
-          double X[8][3], U[8][3], B[8][3];
+          double X[8][3], U[8][3], B[8][3], phi[3];
           ZoneOut o;
           gather_corners(D, D.x, D.u, i, j, k, X, U);
-          zone_state(X, U, D.m[id], D.e[id], 0.0, h->pr, B, &o);
+          if (h->pr.q_kind == 1) mono_phi(h, g, phi);
+          zone_state(X, U, D.m[id], D.e[id], 0.0, h->pr, B, &o,
+                     h->pr.q_kind == 1 ? phi : nullptr);
           if (mask & ORC_F_RHO) out[6][gi] = o.rho;
           if (mask & ORC_F_E) out[7][gi] = D.e[id];
           if (mask & ORC_F_P) out[8][gi] = o.p;

@@ -54,6 +54,7 @@ typedef struct {
   double dt_floor;              /* dt-collapse floor (reading R23): > 0 absolute; 0 = 1e-6 * dt^0;
                                    < 0 = none.  A cycle whose min_z dt_z is below it halts the run
                                    with ORC_EDTMIN (bad_zone -1), unless it ends the run at t_stop */
+  int32_t q_kind;               /* 0: scalar q (reading R7); 1: monotone q (reading R24) */
 } orc_config;
 
 typedef struct {
@@ -91,6 +92,11 @@ void orc_zone_geometry(const double X[8][3], double B[8][3], double *V, double *
 void orc_zone_state(const double X[8][3], const double U[8][3], double m, double e, double hh,
                     double gamma, double q_lin, double q_quad, double cfl, double c_vol,
                     double out[8] /* rho, e_p, p, c, q, P, dt_z, V */);
+
+/* f1 (reading R24): strain rate eps_d and length L_d of one zone along each logical direction,
+   and the monotonic limiter of one direction from the strain rates (em, e0, ep). */
+void orc_zone_strain(const double X[8][3], const double U[8][3], double eps[3], double L[3]);
+double orc_mono_limiter(double em, double e0, double ep);
 
 /* f1 (reading R17): Flanagan-Belytschko viscous hourglass corner forces of one zone, from the
    half-step positions X, velocities U, corner vectors B, V, rho, c and kappa (hydro_oracle.cpp). */
