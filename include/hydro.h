@@ -35,7 +35,7 @@
 extern "C" {
 #endif
 
-#define HYDRO_ABI_VERSION 3
+#define HYDRO_ABI_VERSION 4
 
 typedef struct hydro_ctx hydro_ctx; /* opaque; owned by the library */
 
@@ -132,6 +132,11 @@ typedef struct {
                                    < 0 = no floor.  A cycle whose min_z dt_z falls below it halts
                                    the run with HYDRO_EDTMIN (state = the one after that cycle),
                                    unless that cycle reaches t_stop. */
+  int32_t q_kind;               /* artificial viscosity: 0 = scalar von
+                                   Neumann-Richtmyer + Landshoff q (reading R7, the default);
+                                   1 = monotone q (reading R24: per logical direction, limited by
+                                   the neighbours' strain rates; single rank only, runs the split
+                                   kernels like hg_coef > 0; EINVAL with nranks > 1) */
 } hydro_config;
 
 typedef struct {

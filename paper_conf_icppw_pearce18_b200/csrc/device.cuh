@@ -31,6 +31,8 @@ struct DomView {
   double *mn8;                          // node: 8 / (sum of the <= 8 zone masses around it),
                                         // constant (Lagrangian masses, S7); see k_nodal_mass
   double *mi;                           // zone: 1 / m (0 outside the mesh), constant
+  double *eps;                          // monotone q (R24): 3 zone planes of strain rates of
+                                        // the owned zones (scratch; nullptr unless q_kind 1)
   int32_t dom;                          // global domain index
   int32_t pad_;
 
@@ -46,8 +48,17 @@ struct Phys {
   double gamma, gm1, ggm1, q_lin, q_quad, cfl, c_vol;
   double dt_growth, dt_max, t_stop;
   uint32_t reflect_mask;
-  uint32_t pad_;
+  int32_t q_kind;  // 0 scalar q (reading R7), 1 monotone q (reading R24; split / STRICT paths)
   double hg;  // hourglass kappa (split path only; 0 = off)
+};
+
+// Reading R24 (monotone q): where the strain rate of any global zone lives.  Single rank: every
+// domain is on this GPU.  Owner of global zone g = domain (zown0[g0], zown1[g1], zown2[g2]).
+struct MonoMap {
+  const int32_t *zown[3];  // per axis: domain coordinate of each global zone index
+  const int32_t *slot;     // global domain -> local slot
+  const DomView *views;    // local views (current parity; eps is parity-free)
+  int32_t ndx, ndy;
 };
 
 // Device-resident scalar state of a run (one per rank).  Kernels read t, dt from here so a

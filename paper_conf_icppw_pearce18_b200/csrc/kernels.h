@@ -79,12 +79,17 @@ void launch_init_zones(const DomView &d, int kind, double rho0, double e0, doubl
 // after init, so once per run).
 void launch_nodal_mass(const DomView &d, cudaStream_t s);
 // dt^0 (S2-S6 at x^0 with no predictor) over owned zones -> st->dtz_acc, error flags.
-void launch_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+// M: monotone-q lookup (reading R24; only read when ph.q_kind == 1).
+void launch_dt0(const DomView &d, const Phys &ph, DevState *st, const MonoMap &M,
+                cudaStream_t s);
+// Reading R24: d.eps <- strain rates of the owned zones at x + dt/2 u (at_x: at x).
+void launch_strain(const DomView &d, const DevState *st, int at_x, cudaStream_t s);
 void launch_finalize_init(DevState *st, double dt_first, double dt_init, double dt_max,
                           double t_stop, double t0, double dt_floor, cudaStream_t s);
 
 // Split 3-kernel pipeline (naive, obviously-correct path; HYDRO_FLAG_SPLIT).
-void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, const MonoMap &M,
+                       cudaStream_t s);
 void launch_node_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 void launch_energy_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 
@@ -92,11 +97,14 @@ void launch_energy_split(const DomView &d, const Phys &ph, DevState *st, cudaStr
 // split pipeline in the canonical operation order of SURVEY §8c, bitwise equal to the oracle.
 void launch_strict_init_zones(const DomView &d, int kind, double rho0, double e0, double E,
                               cudaStream_t s);
-void launch_strict_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
-void launch_strict_zone(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
+void launch_strict_dt0(const DomView &d, const Phys &ph, DevState *st, const MonoMap &M,
+                       cudaStream_t s);
+void launch_strict_strain(const DomView &d, const DevState *st, int at_x, cudaStream_t s);
+void launch_strict_zone(const DomView &d, const Phys &ph, DevState *st, const MonoMap &M,
+                        cudaStream_t s);
 void launch_strict_node(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
 void launch_strict_energy(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s);
-void launch_strict_derive(const DomView &d, const Phys &ph, cudaStream_t s);
+void launch_strict_derive(const DomView &d, const Phys &ph, const MonoMap &M, cudaStream_t s);
 
 // TMA descriptors of one domain and parity: the six node-state arrays (x,y,z,u,v,w), the
 // constant nodal 8/mass array and the
@@ -169,6 +177,6 @@ void launch_copy3d(const double *src, int64_t ssx, int64_t ssxy, double *dst, in
                    int64_t dsxy, int ex, int ey, int ez, cudaStream_t s);
 
 // get_fields: derived zone fields (rho, p, q, c, vol) at (x, u) with no predictor into d.aux.
-void launch_derive(const DomView &d, const Phys &ph, cudaStream_t s);
+void launch_derive(const DomView &d, const Phys &ph, const MonoMap &M, cudaStream_t s);
 
 }  // namespace hydro

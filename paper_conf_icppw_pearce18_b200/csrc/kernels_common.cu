@@ -116,7 +116,36 @@ __global__ void k_inv_mass(DomView d, int64_t nz) {
 }
 
 // dt^0: S2-S6 at x^0 with no predictor over owned zones.
-__global__ void k_dt0(DomView d, Phys ph, DevState *st) {
+// Reading R24 (monotone q): the limiter values and the zone's own strain data (phi[3],
+// epsL[6]) of local zone (i,j,k) from its corners; false = scalar q.
+__device__ __forceinline__ bool mono_inputs(const DomView &d, const Phys &ph, const MonoMap &M,
+                                            int i, int j, int k, const double X[8],
+                                            const double Y[8], const double Z[8],
+                                            const double U[8], const double Vv[8],
+                                            const double W[8], double phi[3], double epsL[6]) {
+  if (ph.q_kind != 1) return false;
+  const int64_t g[3] = {d.lo[0] + i, d.lo[1] + j, d.lo[2] + k};
+  mono_phi(M, d.N, g, ph.reflect_mask, phi);
+  zone_strain(X, Y, Z, U, Vv, W, epsL, epsL + 3);
+  return true;
+}
+
+// Reading R24: strain rates of the owned zones at x + hh u (hh = dt/2, or 0 with at_x).
+__global__ void k_strain(DomView d, const DevState *st, int at_x) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int j = blockIdx.y * blockDim.y + threadIdx.y;
+  const int k = blockIdx.z;
+  if (i >= d.n[0] || j >= d.n[1]) return;
+  const double hh = at_x ? 0.0 : 0.5 * st->dt;
+  double X[8], Y[8], Z[8], U[8], Vv[8], W[8], eps[3], L[3];
+  gather(d, i, j, k, hh, X, Y, Z, U, Vv, W);
+  zone_strain(X, Y, Z, U, Vv, W, eps, L);
+  const int64_t id = d.zid(i, j, k);
+#pragma unroll
+  for (int dd = 0; dd < 3; ++dd) d.eps[(int64_t)dd * d.nzone + id] = eps[dd];
+}
+
+__global__ void k_dt0(DomView d, Phys ph, DevState *st, MonoMap M) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   const int j = blockIdx.y * blockDim.y + threadIdx.y;
   const int k = blockIdx.z;
@@ -129,7 +158,10 @@ __global__ void k_dt0(DomView d, Phys ph, DevState *st) {
 #pragma unroll
     for (int l = 0; l < 8; ++l) DV += U[l] * Bx[l] + Vv[l] * By[l] + W[l] * Bz[l];
     const int64_t id = d.zid(i, j, k);
-    const ZoneEos r = zone_eos(V, A2, DV, d.m[id], d.e[id], 0.0, ph);
+    double phi[3], epsL[6];
+    const bool mono = mono_inputs(d, ph, M, i, j, k, X, Y, Z, U, Vv, W, phi, epsL);
+    const ZoneEos r = zone_eos(V, A2, DV, d.m[id], d.e[id], 0.0, ph, mono ? phi : nullptr,
+                               mono ? epsL : nullptr);
     if (!(V > 0.0)) flag_error(st, ERR_TANGLED, global_zone(d, i, j, k));
     dtz = (r.dtz == r.dtz) ? r.dtz : INFINITY;
   }
@@ -161,7 +193,7 @@ __global__ void k_finalize(DevState *st, Phys ph) {
 // ------------------------------------------------------------------ split pipeline
 // K1: S1-S6 for every existing local zone (owned and ghost): P and the 24 corner-vector
 // components to scratch, dt_z min over owned zones.
-__global__ void k_zone_split(DomView d, Phys ph, DevState *st) {
+__global__ void k_zone_split(DomView d, Phys ph, DevState *st, MonoMap M) {
   if (stopped(st)) return;
   const int i = blockIdx.x * blockDim.x + threadIdx.x - 1;
   const int j = blockIdx.y * blockDim.y + threadIdx.y - 1;
@@ -176,7 +208,10 @@ __global__ void k_zone_split(DomView d, Phys ph, DevState *st) {
 #pragma unroll
     for (int l = 0; l < 8; ++l) DV += U[l] * Bx[l] + Vv[l] * By[l] + W[l] * Bz[l];
     const int64_t id = d.zid(i, j, k);
-    const ZoneEos r = zone_eos(V, A2, DV, d.m[id], d.e[id], hh, ph);
+    double phi[3], epsL[6];
+    const bool mono = mono_inputs(d, ph, M, i, j, k, X, Y, Z, U, Vv, W, phi, epsL);
+    const ZoneEos r = zone_eos(V, A2, DV, d.m[id], d.e[id], hh, ph, mono ? phi : nullptr,
+                               mono ? epsL : nullptr);
     d.P[id] = r.P;
     // S5 corner forces f_l = P B_l (+ the f1 hourglass force), 24 planes for K2 and K3
     double Fx[8], Fy[8], Fz[8];
@@ -326,7 +361,7 @@ __global__ void k_halo_copy(const DomView *views, const HaloCopy *chunks) {
 }
 
 // ------------------------------------------------------------------------ outputs
-__global__ void k_derive(DomView d, Phys ph) {
+__global__ void k_derive(DomView d, Phys ph, MonoMap M) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   const int j = blockIdx.y * blockDim.y + threadIdx.y;
   const int k = blockIdx.z;
@@ -338,7 +373,10 @@ __global__ void k_derive(DomView d, Phys ph) {
 #pragma unroll
   for (int l = 0; l < 8; ++l) DV += U[l] * Bx[l] + Vv[l] * By[l] + W[l] * Bz[l];
   const int64_t id = d.zid(i, j, k);
-  const ZoneEos r = zone_eos(V, A2, DV, d.m[id], d.e[id], 0.0, ph);
+  double phi[3], epsL[6];
+  const bool mono = mono_inputs(d, ph, M, i, j, k, X, Y, Z, U, Vv, W, phi, epsL);
+  const ZoneEos r = zone_eos(V, A2, DV, d.m[id], d.e[id], 0.0, ph, mono ? phi : nullptr,
+                             mono ? epsL : nullptr);
   d.aux[0 * d.nzone + id] = r.rho;
   d.aux[1 * d.nzone + id] = r.p;
   d.aux[2 * d.nzone + id] = r.q;
@@ -376,8 +414,12 @@ void launch_nodal_mass(const DomView &d, cudaStream_t s) {
   k_inv_mass<<<(int)std::min<int64_t>((nz + 255) / 256, 4096), 256, 0, s>>>(d, nz);
   k_nodal_mass<<<grid_for(d.n[0] + 1, d.n[1] + 1, d.n[2] + 1), dim3(BX, BY), 0, s>>>(d);
 }
-void launch_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
-  k_dt0<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph, st);
+void launch_strain(const DomView &d, const DevState *st, int at_x, cudaStream_t s) {
+  k_strain<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, st, at_x);
+}
+void launch_dt0(const DomView &d, const Phys &ph, DevState *st, const MonoMap &M,
+                cudaStream_t s) {
+  k_dt0<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph, st, M);
 }
 void launch_finalize_init(DevState *st, double dt_first, double dt_init, double dt_max,
                           double t_stop, double t0, double dt_floor, cudaStream_t s) {
@@ -397,8 +439,10 @@ __global__ void k_reset_clock(DevState *st, double t, double dt, unsigned done) 
 void launch_reset_clock(DevState *st, double t, double dt, unsigned done, cudaStream_t s) {
   k_reset_clock<<<1, 1, 0, s>>>(st, t, dt, done);
 }
-void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
-  k_zone_split<<<grid_for(d.n[0] + 2, d.n[1] + 2, d.n[2] + 2), dim3(BX, BY), 0, s>>>(d, ph, st);
+void launch_zone_split(const DomView &d, const Phys &ph, DevState *st, const MonoMap &M,
+                       cudaStream_t s) {
+  k_zone_split<<<grid_for(d.n[0] + 2, d.n[1] + 2, d.n[2] + 2), dim3(BX, BY), 0, s>>>(d, ph, st,
+                                                                                     M);
 }
 void launch_node_split(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
   k_node_split<<<grid_for(d.n[0] + 1, d.n[1] + 1, d.n[2] + 1), dim3(BX, BY), 0, s>>>(d, ph, st);
@@ -425,8 +469,8 @@ void launch_copy3d(const double *src, int64_t ssx, int64_t ssxy, double *dst, in
   k_copy3d<<<dim3(1, ey, ez), 128, 0, s>>>(src, ssx, ssxy, dst, dsx, dsxy, ex);
 }
 
-void launch_derive(const DomView &d, const Phys &ph, cudaStream_t s) {
-  k_derive<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph);
+void launch_derive(const DomView &d, const Phys &ph, const MonoMap &M, cudaStream_t s) {
+  k_derive<<<grid_for(d.n[0], d.n[1], d.n[2]), dim3(BX, BY), 0, s>>>(d, ph, M);
 }
 
 }  // namespace hydro

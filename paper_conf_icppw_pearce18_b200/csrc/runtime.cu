@@ -98,6 +98,9 @@ struct hydro_ctx {
   int parity = 0;
   bool split = false;
   bool strict = false;  // HYDRO_FLAG_STRICT: the split pipeline in the oracle's operation order
+  // monotone q (reading R24): strain-rate planes per domain and the owner lookup tables
+  MonoMap mono = {};
+  std::vector<void *> mono_mem;
   bool one_kernel = false;
   bool use_graph = true;
   int failed = 0;
@@ -510,12 +513,23 @@ int build_push_tables(hydro_ctx *h) {
   return HYDRO_OK;
 }
 
+// Reading R24: strain rates of every local domain's owned zones (at x_p, or at x with at_x),
+// before any kernel reads a limiter (limiters read their neighbours' owners).
+void launch_strains(hydro_ctx *h, int par, int at_x, cudaStream_t s) {
+  if (h->ph.q_kind != 1) return;
+  for (LocalDom &D : h->doms) {
+    if (h->strict) launch_strict_strain(D.view[par], h->st, at_x, s);
+    else launch_strain(D.view[par], h->st, at_x, s);
+  }
+}
+
 // Split pipeline (plain or STRICT): zone kernels of every domain, the dt / error reduction,
 // then node and energy kernels.
 int enqueue_split(hydro_ctx *h, int par, cudaStream_t s) {
+  launch_strains(h, par, 0, s);
   for (LocalDom &D : h->doms) {
-    if (h->strict) launch_strict_zone(D.view[par], h->ph, h->st, s);
-    else launch_zone_split(D.view[par], h->ph, h->st, s);
+    if (h->strict) launch_strict_zone(D.view[par], h->ph, h->st, h->mono, s);
+    else launch_zone_split(D.view[par], h->ph, h->st, h->mono, s);
   }
   if (h->comm) {
     int rc = comm_dt_min(h->comm, h->st, s);
@@ -690,6 +704,9 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
   if (!valid_phys(cfg)) return set_err(nullptr, HYDRO_EINVAL, "invalid physics parameters");
   if (cfg->init_kind < 0 || cfg->init_kind > 2)
     return set_err(nullptr, HYDRO_EINVAL, "invalid init_kind");
+  if (cfg->q_kind < 0 || cfg->q_kind > 1) return set_err(nullptr, HYDRO_EINVAL, "invalid q_kind");
+  if (cfg->q_kind == 1 && cfg->nranks > 1)  // limiters read zones two layers out (R24)
+    return set_err(nullptr, HYDRO_EINVAL, "monotone q needs a single rank");
   if (cfg->init_kind != HYDRO_INIT_SEDOV)
     for (int f = 0; f < 8; ++f)
       if (!cfg->user[f]) return set_err(nullptr, HYDRO_EINVAL, "USER init needs 8 arrays");
@@ -718,9 +735,12 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
   h->ph.t_stop = cfg->t_stop;
   h->ph.reflect_mask = cfg->reflect_mask;
   h->ph.hg = cfg->hg_coef;
+  h->ph.q_kind = cfg->q_kind;
   // hourglass control (f1) needs per-corner forces, which only the split kernels carry
   h->strict = (cfg->flags & HYDRO_FLAG_STRICT) != 0;
-  h->split = (cfg->flags & HYDRO_FLAG_SPLIT) != 0 || cfg->hg_coef > 0.0 || h->strict;
+  // hourglass control (f1, R17) and the monotone q (f1, R24) run on the split kernels
+  h->split = (cfg->flags & HYDRO_FLAG_SPLIT) != 0 || cfg->hg_coef > 0.0 || h->strict ||
+             cfg->q_kind == 1;
   h->one_kernel = !h->split && (cfg->flags & HYDRO_FLAG_ONE_KERNEL) != 0;
   h->use_graph = (cfg->flags & HYDRO_FLAG_NO_GRAPH) == 0;
   h->device = cfg->device;
@@ -775,6 +795,36 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
            int r = alloc_domain(h, D, h->split);
            if (r) return r;
          }
+         if (h->ph.q_kind == 1) {  // R24: strain planes and owner tables (all domains local)
+           for (LocalDom &D : h->doms) {
+             void *p = nullptr;
+             CK(cudaMalloc(&p, 3 * D.view[0].nzone * sizeof(double)));
+             CK(cudaMemsetAsync(p, 0, 3 * D.view[0].nzone * sizeof(double), h->stream));
+             h->mono_mem.push_back(p);
+             D.view[0].eps = D.view[1].eps = (double *)p;
+           }
+           for (int a = 0; a < 3; ++a) {
+             std::vector<int32_t> own(h->L.N[a]);
+             for (int64_t g = 0; g < h->L.N[a]; ++g) {
+               int d = 0;
+               while (!(h->L.cuts[a][d] <= g && g < h->L.cuts[a][d + 1])) ++d;
+               own[g] = d;
+             }
+             void *p = nullptr;
+             CK(cudaMalloc(&p, own.size() * sizeof(int32_t)));
+             CK(cudaMemcpy(p, own.data(), own.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+             h->mono_mem.push_back(p);
+             h->mono.zown[a] = (const int32_t *)p;
+           }
+           void *p = nullptr;
+           CK(cudaMalloc(&p, h->slot_of_dom.size() * sizeof(int32_t)));
+           CK(cudaMemcpy(p, h->slot_of_dom.data(), h->slot_of_dom.size() * sizeof(int32_t),
+                         cudaMemcpyHostToDevice));
+           h->mono_mem.push_back(p);
+           h->mono.slot = (const int32_t *)p;
+           h->mono.ndx = h->L.nd[0];
+           h->mono.ndy = h->L.nd[1];
+         }
          // device views and intra-GPU halo pairs
          for (int par = 0; par < 2; ++par) {
            CK(cudaMalloc(&h->views_dev[par], sizeof(DomView) * std::max<size_t>(1, h->doms.size())));
@@ -804,6 +854,7 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
              }
            }
          }
+         h->mono.views = h->views_dev[0];  // parity-free fields only (lo, strides, eps)
          // several domains on this GPU: one grouped zone-stage launch covers them all
          // (HYDRO_NO_GROUP=1: one launch per domain, for A/B)
          h->group = h->doms.size() > 1 && !h->split && !h->one_kernel &&
@@ -989,12 +1040,13 @@ int hydro_create(const hydro_config *cfg, hydro_ctx **out) {
                                h->stream);
          }
          for (LocalDom &D : h->doms) launch_nodal_mass(D.view[0], h->stream);
+         launch_strains(h, 0, 1, h->stream);
          for (LocalDom &D : h->doms) {
            if (h->strict) {  // dt^0, then the other parity := this one (node kernel, dt = 0)
-             launch_strict_dt0(D.view[0], h->ph, h->st, h->stream);
+             launch_strict_dt0(D.view[0], h->ph, h->st, h->mono, h->stream);
              launch_strict_node(D.view[0], h->ph, h->st, h->stream);
            } else {
-             launch_dt0(D.view[0], h->ph, h->st, h->stream);
+             launch_dt0(D.view[0], h->ph, h->st, h->mono, h->stream);
            }
          }
          if (h->comm) {
@@ -1233,9 +1285,10 @@ int hydro_get_box(hydro_ctx *h, const int64_t lo[3], const int64_t hi[3], uint32
   const int par = h->parity;
   const bool derived = (mask & (HYDRO_F_RHO | HYDRO_F_P | HYDRO_F_Q | HYDRO_F_C | HYDRO_F_VOL)) != 0;
   if (derived)
+    launch_strains(h, par, 1, h->stream);
     for (LocalDom &D : h->doms) {
-      if (h->strict) launch_strict_derive(D.view[par], h->ph, h->stream);
-      else launch_derive(D.view[par], h->ph, h->stream);
+      if (h->strict) launch_strict_derive(D.view[par], h->ph, h->mono, h->stream);
+      else launch_derive(D.view[par], h->ph, h->mono, h->stream);
     }
   const int64_t bn[3] = {hi[0] - lo[0] + 1, hi[1] - lo[1] + 1, hi[2] - lo[2] + 1};
   const int64_t bz[3] = {hi[0] - lo[0], hi[1] - lo[1], hi[2] - lo[2]};
@@ -1612,6 +1665,7 @@ int hydro_destroy(hydro_ctx *h) {
     if (h->flag_ev[k]) cudaEventDestroy(h->flag_ev[k]);
   if (h->flag_host) cudaFreeHost(h->flag_host);
   if (h->pcopy_dev) cudaFree(h->pcopy_dev);
+  for (void *p : h->mono_mem) cudaFree(p);
   for (int p = 0; p < 2; ++p) {
     if (h->graph[p]) cudaGraphExecDestroy(h->graph[p]);
     if (h->graphk[p]) cudaGraphExecDestroy(h->graphk[p]);

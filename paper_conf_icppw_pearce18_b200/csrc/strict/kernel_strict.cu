@@ -94,9 +94,39 @@ struct SOut {
   double rho, p, c, q, P, dtz, V;
 };
 
+// Reading R24 strain rates in the written order (face sums over corners in ascending l, each
+// sum initialised by its first term; dx = 0.25 (sum+ - sum-); L^2 = dx.dx; eps = du.dx / L^2).
+__device__ void s_strain(const double X[24], const double U[24], double eps[3], double L[3]) {
+#pragma unroll
+  for (int dd = 0; dd < 3; ++dd) {
+    double xs[2][3], us[2][3];
+    bool first[2] = {true, true};
+#pragma unroll
+    for (int l = 0; l < 8; ++l) {
+      const int side = (l >> dd) & 1;
+#pragma unroll
+      for (int k = 0; k < 3; ++k) {
+        xs[side][k] = first[side] ? X[3 * l + k] : xs[side][k] + X[3 * l + k];
+        us[side][k] = first[side] ? U[3 * l + k] : us[side][k] + U[3 * l + k];
+      }
+      first[side] = false;
+    }
+    double dx[3], du[3];
+#pragma unroll
+    for (int k = 0; k < 3; ++k) {
+      dx[k] = 0.25 * (xs[1][k] - xs[0][k]);
+      du[k] = 0.25 * (us[1][k] - us[0][k]);
+    }
+    const double L2 = sdot(dx, dx);
+    eps[dd] = sdot(du, dx) / L2;
+    L[dd] = sqrt(L2);
+  }
+}
+
 // S2 (DV, rho, D) + S3 + S4 + S6 of one zone; B is returned for S5.
 __device__ void s_zone_state(const double X[24], const double U[24], double m, double e,
-                             double hh, const Phys &ph, double B[24], SOut &o) {
+                             double hh, const Phys &ph, double B[24], SOut &o,
+                             const double *phi = nullptr) {
   double V, L;
   s_geometry(X, B, V, L);
   double DV = 0.0;
@@ -115,9 +145,19 @@ __device__ void s_zone_state(const double X[24], const double U[24], double m, d
   const double p = (ph.gm1 * rho) * eppos;
   const double c = sqrt(ph.ggm1 * eppos);
   double qr = 0.0;
-  if (D < 0.0) {
+  if (D < 0.0 && !phi) {
     const double s = L * (-D);
     qr = s * ((ph.q_quad * s) + (ph.q_lin * c));
+  } else if (D < 0.0) {  // reading R24
+    double eps[3], Ld[3];
+    s_strain(X, U, eps, Ld);
+#pragma unroll
+    for (int dd = 0; dd < 3; ++dd) {
+      const double dv = Ld[dd] * smax(-eps[dd], 0.0);
+      const double t = ((ph.q_quad * dv) * dv) * (1.0 - phi[dd] * phi[dd]) +
+                       ((ph.q_lin * c) * dv) * (1.0 - phi[dd]);
+      qr = (dd == 0) ? t : qr + t;
+    }
   }
   const double q = rho * qr;
   const double sig = sqrt(c * c + 2.0 * qr);
@@ -233,6 +273,16 @@ __device__ __forceinline__ void s_gather(const DomView &d, int i, int j, int k, 
   }
 }
 
+// R24 limiter inputs of local zone (i,j,k) (mono_phi: owner lookups + the written limiter)
+__device__ __forceinline__ const double *s_phi(const DomView &d, const Phys &ph,
+                                               const MonoMap &M, int i, int j, int k,
+                                               double phi[3]) {
+  if (ph.q_kind != 1) return nullptr;
+  const int64_t g[3] = {d.lo[0] + i, d.lo[1] + j, d.lo[2] + k};
+  mono_phi(M, d.N, g, ph.reflect_mask, phi);
+  return phi;
+}
+
 __device__ __forceinline__ void s_flag(DevState *st, unsigned bits, int64_t gz) {
   atomicOr(&st->err, bits);
   atomicMin(&st->bad_zone, (unsigned long long)gz);
@@ -269,8 +319,21 @@ __global__ void k_s_init_zones(DomView d, int kind, double rho0, double e0, doub
   }
 }
 
+// R24: strain rates of the owned zones at x + hh u (at_x: hh = 0).
+__global__ void k_s_strain(DomView d, const DevState *st, int at_x) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int j = blockIdx.y * blockDim.y + threadIdx.y;
+  const int k = blockIdx.z;
+  if (i >= d.n[0] || j >= d.n[1]) return;
+  double X[24], U[24], eps[3], L[3];
+  s_gather(d, i, j, k, at_x ? 0.0 : 0.5 * st->dt, false, X, U);
+  s_strain(X, U, eps, L);
+  const int64_t id = d.zid(i, j, k);
+  for (int dd = 0; dd < 3; ++dd) d.eps[(int64_t)dd * d.nzone + id] = eps[dd];
+}
+
 // dt^0: S2-S6 at x^0, no predictor, owned zones; also x^{n+1} := x (the other parity).
-__global__ void k_s_dt0(DomView d, Phys ph, DevState *st) {
+__global__ void k_s_dt0(DomView d, Phys ph, DevState *st, MonoMap M) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   const int j = blockIdx.y * blockDim.y + threadIdx.y;
   const int k = blockIdx.z;
@@ -280,7 +343,8 @@ __global__ void k_s_dt0(DomView d, Phys ph, DevState *st) {
     SOut o;
     s_gather(d, i, j, k, 0.0, false, X, U);
     const int64_t id = d.zid(i, j, k);
-    s_zone_state(X, U, d.m[id], d.e[id], 0.0, ph, B, o);
+    double phi[3];
+    s_zone_state(X, U, d.m[id], d.e[id], 0.0, ph, B, o, s_phi(d, ph, M, i, j, k, phi));
     if (!(o.V > 0.0)) s_flag(st, ERR_TANGLED, s_gzone(d, i, j, k));
     dtz = (o.dtz == o.dtz) ? o.dtz : INFINITY;
   }
@@ -289,7 +353,7 @@ __global__ void k_s_dt0(DomView d, Phys ph, DevState *st) {
 
 // K1 (S1-S6): every existing zone of the domain and its ghost ring: corner forces
 // f_l = P B_l (+ f_hg_l) into the 24 planes of d.B; dt_z over owned zones.
-__global__ void k_s_zone(DomView d, Phys ph, DevState *st) {
+__global__ void k_s_zone(DomView d, Phys ph, DevState *st, MonoMap M) {
   if ((st->halted | st->done) != 0u) return;
   const int i = blockIdx.x * blockDim.x + threadIdx.x - 1;
   const int j = blockIdx.y * blockDim.y + threadIdx.y - 1;
@@ -301,7 +365,8 @@ __global__ void k_s_zone(DomView d, Phys ph, DevState *st) {
     SOut o;
     s_gather(d, i, j, k, hh, false, X, U);
     const int64_t id = d.zid(i, j, k);
-    s_zone_state(X, U, d.m[id], d.e[id], hh, ph, B, o);
+    double phi[3];
+    s_zone_state(X, U, d.m[id], d.e[id], hh, ph, B, o, s_phi(d, ph, M, i, j, k, phi));
     double f[24];
 #pragma unroll
     for (int c = 0; c < 24; ++c) f[c] = o.P * B[c];
@@ -401,7 +466,7 @@ __global__ void k_s_energy(DomView d, Phys ph, DevState *st) {
 }
 
 // Outputs: rho, p, q, c, V by S2-S4 at (x, u) with e_p = e.
-__global__ void k_s_derive(DomView d, Phys ph) {
+__global__ void k_s_derive(DomView d, Phys ph, MonoMap M) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   const int j = blockIdx.y * blockDim.y + threadIdx.y;
   const int k = blockIdx.z;
@@ -410,7 +475,8 @@ __global__ void k_s_derive(DomView d, Phys ph) {
   SOut o;
   s_gather(d, i, j, k, 0.0, false, X, U);
   const int64_t id = d.zid(i, j, k);
-  s_zone_state(X, U, d.m[id], d.e[id], 0.0, ph, B, o);
+  double phi[3];
+  s_zone_state(X, U, d.m[id], d.e[id], 0.0, ph, B, o, s_phi(d, ph, M, i, j, k, phi));
   d.aux[0 * d.nzone + id] = o.rho;
   d.aux[1 * d.nzone + id] = o.p;
   d.aux[2 * d.nzone + id] = o.q;
@@ -427,11 +493,16 @@ void launch_strict_init_zones(const DomView &d, int kind, double rho0, double e0
   k_s_init_zones<<<sgrid(d.n[0] + 2, d.n[1] + 2, d.n[2] + 2), dim3(SBX, SBY), 0, s>>>(
       d, kind, rho0, e0, E);
 }
-void launch_strict_dt0(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
-  k_s_dt0<<<sgrid(d.n[0], d.n[1], d.n[2]), dim3(SBX, SBY), 0, s>>>(d, ph, st);
+void launch_strict_dt0(const DomView &d, const Phys &ph, DevState *st, const MonoMap &M,
+                       cudaStream_t s) {
+  k_s_dt0<<<sgrid(d.n[0], d.n[1], d.n[2]), dim3(SBX, SBY), 0, s>>>(d, ph, st, M);
 }
-void launch_strict_zone(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
-  k_s_zone<<<sgrid(d.n[0] + 2, d.n[1] + 2, d.n[2] + 2), dim3(SBX, SBY), 0, s>>>(d, ph, st);
+void launch_strict_strain(const DomView &d, const DevState *st, int at_x, cudaStream_t s) {
+  k_s_strain<<<sgrid(d.n[0], d.n[1], d.n[2]), dim3(SBX, SBY), 0, s>>>(d, st, at_x);
+}
+void launch_strict_zone(const DomView &d, const Phys &ph, DevState *st, const MonoMap &M,
+                        cudaStream_t s) {
+  k_s_zone<<<sgrid(d.n[0] + 2, d.n[1] + 2, d.n[2] + 2), dim3(SBX, SBY), 0, s>>>(d, ph, st, M);
 }
 void launch_strict_node(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
   k_s_node<<<sgrid(d.n[0] + 1, d.n[1] + 1, d.n[2] + 1), dim3(SBX, SBY), 0, s>>>(d, ph, st);
@@ -439,8 +510,8 @@ void launch_strict_node(const DomView &d, const Phys &ph, DevState *st, cudaStre
 void launch_strict_energy(const DomView &d, const Phys &ph, DevState *st, cudaStream_t s) {
   k_s_energy<<<sgrid(d.n[0], d.n[1], d.n[2]), dim3(SBX, SBY), 0, s>>>(d, ph, st);
 }
-void launch_strict_derive(const DomView &d, const Phys &ph, cudaStream_t s) {
-  k_s_derive<<<sgrid(d.n[0], d.n[1], d.n[2]), dim3(SBX, SBY), 0, s>>>(d, ph);
+void launch_strict_derive(const DomView &d, const Phys &ph, const MonoMap &M, cudaStream_t s) {
+  k_s_derive<<<sgrid(d.n[0], d.n[1], d.n[2]), dim3(SBX, SBY), 0, s>>>(d, ph, M);
 }
 
 }  // namespace hydro

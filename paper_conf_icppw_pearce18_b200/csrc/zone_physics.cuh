@@ -144,9 +144,73 @@ struct ZoneEos {
   double rho, p, c, q, P, dtz;
 };
 
-// S2 (rho, D) + S3 + S4 + S6 given V, L = 2V/sqrt(A2max_unscaled), DV = sum u.B.
+// f1 / reading R24 (monotone q): strain rate eps_d = (du_d . dx_d)/|dx_d|^2 and length
+// L_d = |dx_d| of a zone along each logical direction d, from the face-centre differences dx_d,
+// du_d (corners with bit d set minus those without, / 4).
+__device__ __forceinline__ void zone_strain(const double X[8], const double Y[8],
+                                            const double Z[8], const double U[8],
+                                            const double Vv[8], const double W[8],
+                                            double eps[3], double L[3]) {
+#pragma unroll
+  for (int dd = 0; dd < 3; ++dd) {
+    double dx = 0.0, dy = 0.0, dz = 0.0, du = 0.0, dv = 0.0, dw = 0.0;
+#pragma unroll
+    for (int l = 0; l < 8; ++l) {
+      const double sg = ((l >> dd) & 1) ? 0.25 : -0.25;
+      dx = fma(sg, X[l], dx); dy = fma(sg, Y[l], dy); dz = fma(sg, Z[l], dz);
+      du = fma(sg, U[l], du); dv = fma(sg, Vv[l], dv); dw = fma(sg, W[l], dw);
+    }
+    const double L2 = dx * dx + dy * dy + dz * dz;
+    eps[dd] = (du * dx + dv * dy + dw * dz) / L2;
+    L[dd] = sqrt(L2);
+  }
+}
+
+// Reading R24: phi = max(0, min((r- + r+)/2, 2 r-, 2 r+, 1)), r = neighbour / own strain rate.
+__device__ __forceinline__ double mono_limiter(double em, double e0, double ep) {
+  if (e0 == 0.0) return 1.0;
+  const double rm = em / e0, rp = ep / e0;
+  double phi = 0.5 * (rm + rp);
+  phi = (2.0 * rm < phi) ? 2.0 * rm : phi;
+  phi = (2.0 * rp < phi) ? 2.0 * rp : phi;
+  phi = (1.0 < phi) ? 1.0 : phi;
+  return (phi < 0.0) ? 0.0 : phi;
+}
+
+// Strain rate eps_d of global zone (g0, g1, g2), read from its owner domain on this GPU.
+__device__ __forceinline__ double mono_eps(const MonoMap &M, int64_t g0, int64_t g1, int64_t g2,
+                                           int dd) {
+  const int dom = (M.zown[2][g2] * M.ndy + M.zown[1][g1]) * M.ndx + M.zown[0][g0];
+  const DomView &v = M.views[M.slot[dom]];
+  const int64_t id = v.zid((int)(g0 - v.lo[0]), (int)(g1 - v.lo[1]), (int)(g2 - v.lo[2]));
+  return v.eps[(int64_t)dd * v.nzone + id];
+}
+
+// Reading R24: the three limiter values of global zone g (a neighbour outside the mesh mirrors
+// the zone at a reflecting wall and is unstrained at a free boundary).
+__device__ __forceinline__ void mono_phi(const MonoMap &M, const int32_t N[3], const int64_t g[3],
+                                         uint32_t reflect_mask, double phi[3]) {
+#pragma unroll
+  for (int dd = 0; dd < 3; ++dd) {
+    const double e0 = mono_eps(M, g[0], g[1], g[2], dd);
+    int64_t gm[3] = {g[0], g[1], g[2]}, gp[3] = {g[0], g[1], g[2]};
+    gm[dd] -= 1;
+    gp[dd] += 1;
+    const double em = gm[dd] >= 0 ? mono_eps(M, gm[0], gm[1], gm[2], dd)
+                      : ((reflect_mask >> (2 * dd)) & 1u) ? e0 : 0.0;
+    const double ep = gp[dd] < N[dd] ? mono_eps(M, gp[0], gp[1], gp[2], dd)
+                      : ((reflect_mask >> (2 * dd + 1)) & 1u) ? e0 : 0.0;
+    phi[dd] = mono_limiter(em, e0, ep);
+  }
+}
+
+// S2 (rho, D) + S3 + S4 + S6 given V, L = 2V/sqrt(A2max_unscaled), DV = sum u.B.  phi / epsL
+// (monotone q, R24): the zone's limiter values and its own strain rates eps[3] and lengths
+// epsL[3..5]; nullptr = the scalar q of R7.
 __device__ __forceinline__ ZoneEos zone_eos(double V, double A2max, double DV, double m,
-                                            double e, double hh, const Phys &ph) {
+                                            double e, double hh, const Phys &ph,
+                                            const double *phi = nullptr,
+                                            const double *epsL = nullptr) {
   ZoneEos r;
   const double L = 2.0 * V / sqrt(A2max);
   const double inv = 1.0 / V;
@@ -158,9 +222,15 @@ __device__ __forceinline__ ZoneEos zone_eos(double V, double A2max, double DV, d
   const double p = ph.gm1 * rho * eppos;
   const double c = sqrt(ph.ggm1 * eppos);
   double qr = 0.0;
-  if (D < 0.0) {
+  if (D < 0.0 && !phi) {
     const double s = -L * D;
     qr = s * (ph.q_quad * s + ph.q_lin * c);
+  } else if (D < 0.0) {
+#pragma unroll
+    for (int dd = 0; dd < 3; ++dd) {
+      const double dv = epsL[3 + dd] * fmax(-epsL[dd], 0.0);
+      qr += (ph.q_quad * dv) * dv * (1.0 - phi[dd] * phi[dd]) + (ph.q_lin * c) * dv * (1.0 - phi[dd]);
+    }
   }
   r.rho = rho;
   r.p = p;

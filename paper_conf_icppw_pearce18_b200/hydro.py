@@ -22,7 +22,7 @@ LIB_PATH = os.environ.get("HYDRO_LIB") or os.path.join(_HERE, "libhydro_b200.so"
 NODE_FIELDS = ("x", "y", "z", "u", "v", "w")
 ZONE_FIELDS = ("rho", "e", "p", "q", "c", "vol", "mass")
 ALL_FIELDS = NODE_FIELDS + ZONE_FIELDS
-ABI_VERSION = 3
+ABI_VERSION = 4
 FLAG_NO_GRAPH = 1 << 0
 FLAG_SPLIT = 1 << 1
 FLAG_ONE_KERNEL = 1 << 2
@@ -58,6 +58,7 @@ class HydroConfigC(C.Structure):
         ("flags", C.c_uint64),
         ("hg_coef", C.c_double),
         ("dt_floor", C.c_double),
+        ("q_kind", C.c_int32),
     ]
 
 
@@ -168,6 +169,8 @@ class HydroConfig:
                                   # the split kernels
     dt_floor: float = 0.0         # dt-collapse floor (reading R23): > 0 absolute, 0 = 1e-6 dt^0,
                                   # < 0 none; below it a run halts with EDTMIN
+    q: str = "scalar"             # artificial viscosity: "scalar" (reading R7) or "monotone"
+                                  # (reading R24; single rank, split kernels)
     comm_self: bool = False       # nranks == 1: create a one-rank NCCL communicator anyway
                                   # (HYDRO_FLAG_COMM_SELF; exercises the NCCL path on one GPU)
 
@@ -204,6 +207,7 @@ def _cfg_struct(cfg: HydroConfig, keep: list, comm_id: Optional[bytes] = None) -
         setattr(c, k, float(getattr(cfg, k)))
     c.reflect_mask = int(cfg.reflect_mask)
     c.init_kind = {"sedov": 0, "user": 1, "user_mass": 2}[cfg.init]
+    c.q_kind = {"scalar": 0, "monotone": 1}[cfg.q]
     if cfg.init != "sedov":
         names = ("x", "y", "z", "u", "v", "w", "rho" if cfg.init == "user" else "mass", "e")
         for f, nm in enumerate(names):

@@ -27,7 +27,7 @@ def test_library_exports_every_declared_symbol():
     lib = ctypes.CDLL(LIB_PATH)
     missing = [n for n in names if not hasattr(lib, n)]
     assert not missing, missing
-    assert load_library().hydro_abi_version() == 3
+    assert load_library().hydro_abi_version() == 4
 
 
 def parse(buf):
