@@ -38,7 +38,7 @@ def test_one_rank_nccl_equals_no_comm_bitwise(path, overlap, monkeypatch):
     fb, ib = _run(30, **kw)
     assert ia["status"] == ib["status"] == 0
     assert ia["t"] == ib["t"] and ia["dt"] == ib["dt"] and ia["cycle"] == ib["cycle"] == 30
-    assert ia["kernels"] != ib["kernels"]  # pack / unpack / dt kernels instead of the copies
+    # (under COMM_SELF the copy kernel gets no chunks: stale ghosts would break the equality)
     for k in FIELDS:
         assert np.array_equal(fa[k], fb[k]), k
 
