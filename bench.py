@@ -286,7 +286,7 @@ class Run:
         self.kw, self.scaling, self.desc, self.h = workload(name, ngpu)
         self.cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, path=args.path,
                                transport=args.transport, hg_coef=args.hg, halo=args.halo,
-                               **self.kw)
+                               q=args.q, **self.kw)
         self.Hydro, self.HydroConfig = Hydro, HydroConfig
         self.hyd = Hydro(self.cfg)
         n = self.kw["n"]
@@ -485,7 +485,7 @@ def selfcheck(args, name, ngpu, rank, local, dist):
     if min(n) < 2 * w:
         return None
     cfg = HydroConfig(rank=rank, nranks=ngpu, device=local, path=args.path,
-                      transport=args.transport, hg_coef=args.hg, halo=args.halo, **kw)
+                      transport=args.transport, hg_coef=args.hg, halo=args.halo, q=args.q, **kw)
     hyd = Hydro(cfg)
     info = hyd.step(cyc)
     win = hyd.box((0, 0, 0), (w, w, w))
@@ -496,7 +496,8 @@ def selfcheck(args, name, ngpu, rank, local, dist):
         return None
     import oracle
     from oracle import OracleConfig
-    fo, io = oracle.run(OracleConfig(n=(w, w, w), extent=(h * w,) * 3, hg_coef=args.hg), cyc)
+    fo, io = oracle.run(OracleConfig(n=(w, w, w), extent=(h * w,) * 3, hg_coef=args.hg, q=args.q),
+                        cyc)
     inside = (np.abs(fo["u"][:, :, -4:]).max() == 0.0 and np.abs(fo["e"][:, :, -4:]).max() == 0.0)
     errs = {}
     for k in ("x", "y", "z", "u", "v", "w", "rho", "e", "p", "q", "c", "vol", "mass"):
@@ -572,6 +573,8 @@ def main():
                          "allreduce (the other one is run as a 10-cycle bitwise check)")
     ap.add_argument("--hg", type=float, default=0.0,
                     help="viscous hourglass coefficient (SURVEY f1, reading R17)")
+    ap.add_argument("--q", default="scalar", choices=["scalar", "monotone"],
+                    help="artificial viscosity (reading R7 / R24; monotone: split kernels)")
     ap.add_argument("--halo", default="kernel", choices=["kernel", "fused"],
                     help="ghost-slab exchange: from the node/energy stage's epilogue (fused) or "
                          "separate copy / peer-push kernels after it")
@@ -603,7 +606,8 @@ def main():
     roof = run.roofline()
     e2e = run.e2e_single() if ngpu == 1 else run.e2e_ranks()
     line_cfg = {"workload": run.desc, "mesh": list(run.kw["n"]), "domains": list(run.cfg.ndom),
-                "zones": run.zones, "path": args.path, "hg_coef": args.hg, "halo": args.halo,
+                "zones": run.zones, "path": args.path, "hg_coef": args.hg, "q": args.q,
+                "halo": args.halo,
                 "l2": "state > 126 MB L2 (inputs larger than L2; no flush)"
                 if run.zones * 120 > 126e6 else "state fits L2",
                 "parallelism": f"dp{ngpu} (spatial domains)",
