@@ -249,7 +249,9 @@ def run_reference(args):
     # bounded sample: the whole mesh if a step is cheap, else a 64^3 Sedov corner box of the
     # workload's zone size per step
     per_cycle_s = zones / 3.0e6
-    whole = per_cycle_s * (args.steps + args.warmup) < 150
+    # (the whole mesh only up to configs[1]'s 128^3: the oracle needs ~350 B of host memory per
+    # zone, ~47 GB at 512^3)
+    whole = zones <= 2_200_000 and per_cycle_s * (args.steps + args.warmup) < 150
     sample_n = n if whole else (64, 64, 64)
     sz = sample_n[0] * sample_n[1] * sample_n[2]
     o = oracle.Oracle(OracleConfig(n=sample_n, extent=kw.get("extent", (1.2,) * 3) if whole
