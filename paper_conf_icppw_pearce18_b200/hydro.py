@@ -429,7 +429,8 @@ class Hydro:
 
     def fields(self, names: Sequence[str] = ALL_FIELDS,
                out: Optional[Dict[str, np.ndarray]] = None) -> Dict[str, np.ndarray]:
-        """Global fields; ``out`` may supply caller-owned (e.g. pinned) arrays to fill."""
+        """Global fields; ``out`` may supply caller-owned (e.g. pinned) arrays to fill.  With
+        nranks > 1 a collective that assembles them on rank 0 (``_combine``)."""
         nx, ny, nz = (int(v) for v in self.cfg.n)
         out, ptrs, mask = self._arrays(names, (nz + 1, ny + 1, nx + 1), (nz, ny, nx), given=out)
         rc = self._L.hydro_get_fields(self._h, mask, ptrs)
@@ -454,6 +455,10 @@ class Hydro:
         return out
 
     def _combine(self, out):
+        """nranks > 1: every global entry is written by exactly one rank (the rest are zero), so a
+        sum to rank 0 assembles the global arrays there (collective; rank 0 returns them, the
+        other ranks return their own partial arrays).  Rank-local data without any global
+        array: pack_domain / hydro_get_box of the owned domains."""
         import torch
         import torch.distributed as dist
         res = {}
@@ -461,8 +466,8 @@ class Hydro:
             t = torch.from_numpy(v)
             if dist.get_backend(self._group) == "nccl":
                 t = t.cuda()
-            dist.all_reduce(t, group=self._group)  # each entry is written by exactly one rank
-            res[k] = t.cpu().numpy()
+            dist.reduce(t, dst=0, group=self._group)
+            res[k] = t.cpu().numpy() if self.cfg.rank == 0 else v
         return res
 
     # ------------------------------------------------------------ domain migration (f2)
