@@ -243,11 +243,15 @@ int comm_wait(Comm *c, cudaStream_t s, double timeout_s, std::string *err) {
       *err = std::string("stream: ") + cudaGetErrorString(q);
       return HYDRO_ECUDA;
     }
-    ncclResult_t ae = ncclSuccess, ae2 = ncclSuccess;
-    if (c->dtcomm && (ncclCommGetAsyncError(c->dtcomm, &ae2) != ncclSuccess || ae2 != ncclSuccess))
-      ae = ae2 != ncclSuccess ? ae2 : ncclInternalError;
-    if (ae != ncclSuccess || ncclCommGetAsyncError(c->nccl, &ae) != ncclSuccess ||
-        ae != ncclSuccess) {
+    // asynchronous error of either communicator (a failing query counts as an error too)
+    auto async_error = [](ncclComm_t comm) {
+      ncclResult_t r = ncclSuccess;
+      if (ncclCommGetAsyncError(comm, &r) != ncclSuccess) return ncclInternalError;
+      return r;
+    };
+    ncclResult_t ae = async_error(c->nccl);
+    if (ae == ncclSuccess && c->dtcomm) ae = async_error(c->dtcomm);
+    if (ae != ncclSuccess) {
       *err = std::string("NCCL asynchronous error: ") + ncclGetErrorString(ae);
       if (c->dtcomm) ncclCommAbort(c->dtcomm);
       ncclCommAbort(c->nccl);
