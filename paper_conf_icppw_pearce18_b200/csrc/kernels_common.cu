@@ -125,7 +125,7 @@ __device__ __forceinline__ bool mono_inputs(const DomView &d, const Phys &ph, co
                                             const double W[8], double phi[3], double epsL[6]) {
   if (ph.q_kind != 1) return false;
   const int64_t g[3] = {d.lo[0] + i, d.lo[1] + j, d.lo[2] + k};
-  mono_phi(M, d.N, g, ph.reflect_mask, phi);
+  mono_phi(M, d, g, ph.reflect_mask, phi);
   zone_strain(X, Y, Z, U, Vv, W, epsL, epsL + 3);
   return true;
 }

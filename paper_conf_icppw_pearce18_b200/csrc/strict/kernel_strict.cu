@@ -279,7 +279,7 @@ __device__ __forceinline__ const double *s_phi(const DomView &d, const Phys &ph,
                                                double phi[3]) {
   if (ph.q_kind != 1) return nullptr;
   const int64_t g[3] = {d.lo[0] + i, d.lo[1] + j, d.lo[2] + k};
-  mono_phi(M, d.N, g, ph.reflect_mask, phi);
+  mono_phi(M, d, g, ph.reflect_mask, phi);
   return phi;
 }
 

@@ -177,9 +177,13 @@ __device__ __forceinline__ double mono_limiter(double em, double e0, double ep) 
   return (phi < 0.0) ? 0.0 : phi;
 }
 
-// Strain rate eps_d of global zone (g0, g1, g2), read from its owner domain on this GPU.
-__device__ __forceinline__ double mono_eps(const MonoMap &M, int64_t g0, int64_t g1, int64_t g2,
-                                           int dd) {
+// Strain rate eps_d of global zone (g0, g1, g2), read from its owner domain on this GPU: the
+// calling domain `self` itself when it owns the zone (one load), else through the owner tables.
+__device__ __forceinline__ double mono_eps(const MonoMap &M, const DomView &self, int64_t g0,
+                                           int64_t g1, int64_t g2, int dd) {
+  const int64_t l0 = g0 - self.lo[0], l1 = g1 - self.lo[1], l2 = g2 - self.lo[2];
+  if (l0 >= 0 && l0 < self.n[0] && l1 >= 0 && l1 < self.n[1] && l2 >= 0 && l2 < self.n[2])
+    return self.eps[(int64_t)dd * self.nzone + self.zid((int)l0, (int)l1, (int)l2)];
   const int dom = (M.zown[2][g2] * M.ndy + M.zown[1][g1]) * M.ndx + M.zown[0][g0];
   const DomView &v = M.views[M.slot[dom]];
   const int64_t id = v.zid((int)(g0 - v.lo[0]), (int)(g1 - v.lo[1]), (int)(g2 - v.lo[2]));
@@ -188,17 +192,18 @@ __device__ __forceinline__ double mono_eps(const MonoMap &M, int64_t g0, int64_t
 
 // Reading R24: the three limiter values of global zone g (a neighbour outside the mesh mirrors
 // the zone at a reflecting wall and is unstrained at a free boundary).
-__device__ __forceinline__ void mono_phi(const MonoMap &M, const int32_t N[3], const int64_t g[3],
-                                         uint32_t reflect_mask, double phi[3]) {
+__device__ __forceinline__ void mono_phi(const MonoMap &M, const DomView &self,
+                                         const int64_t g[3], uint32_t reflect_mask,
+                                         double phi[3]) {
 #pragma unroll
   for (int dd = 0; dd < 3; ++dd) {
-    const double e0 = mono_eps(M, g[0], g[1], g[2], dd);
+    const double e0 = mono_eps(M, self, g[0], g[1], g[2], dd);
     int64_t gm[3] = {g[0], g[1], g[2]}, gp[3] = {g[0], g[1], g[2]};
     gm[dd] -= 1;
     gp[dd] += 1;
-    const double em = gm[dd] >= 0 ? mono_eps(M, gm[0], gm[1], gm[2], dd)
+    const double em = gm[dd] >= 0 ? mono_eps(M, self, gm[0], gm[1], gm[2], dd)
                       : ((reflect_mask >> (2 * dd)) & 1u) ? e0 : 0.0;
-    const double ep = gp[dd] < N[dd] ? mono_eps(M, gp[0], gp[1], gp[2], dd)
+    const double ep = gp[dd] < self.N[dd] ? mono_eps(M, self, gp[0], gp[1], gp[2], dd)
                       : ((reflect_mask >> (2 * dd + 1)) & 1u) ? e0 : 0.0;
     phi[dd] = mono_limiter(em, e0, ep);
   }
