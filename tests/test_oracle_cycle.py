@@ -252,6 +252,8 @@ def test_sedov_shock_radius_96_cubed_with_hourglass_control():
 
 
 @pytest.mark.slow
+@pytest.mark.skipif(os.environ.get("HYDRO_SLOW") != "1",
+                    reason="37 s; the refined-mesh pin is the 64^3 one (HYDRO_SLOW=1 runs it)")
 def test_sedov_shock_radius_48_cubed():
     n = 48
     cfg = OracleConfig(n=(n, n, n), t_stop=0.3)
